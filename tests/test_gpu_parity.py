@@ -1,0 +1,243 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE.json north_star): grids, samples, indices and the hash
+bit-exact; macroscopic XS within 1e-12 relative (expected exactly equal, reading R8).
+Sizes: tiny in full for every grid type x search variant x sort mode; small in full
+(hash) + sampled outputs; large / large-U / XL at BASELINE sizes on sampled outputs
+and prefix hashes, in the launch configuration bench.py times."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from xs_workloads import GRID_SEED, LOOKUP_SEED, WORKLOADS  # noqa: E402
+
+SEARCHES = ["M", "U1", "U2", "U4", "U8", "B", "M2", "M4", "M8"]
+SORTS = ["none", "material", "material_energy"]
+RTOL = 1e-12
+
+
+@pytest.fixture(scope="module")
+def xs():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_cgo_murtovigplls24_b200 as pkg
+    return pkg
+
+
+@pytest.fixture(scope="module")
+def tiny(xs, oracle_mod):
+    out = {}
+    for gt in (0, 1, 2):
+        g = xs.Grid(68, 1000, gt, GRID_SEED)
+        P = oracle_mod.Problem(68, 1000, gt, GRID_SEED)
+        ref = P.run_range(LOOKUP_SEED, 0, 100_000, macro=True, mat=True, q=True, idx=True)
+        out[gt] = (g, P, ref)
+    yield out
+    for g, _, _ in out.values():
+        g.close()
+
+
+def _macro_close(a, b):
+    a = np.asarray(a)
+    b = np.asarray(b)
+    err = np.abs(a - b) / np.maximum(np.abs(b), 1e-300)
+    return float(err.max()) if err.size else 0.0
+
+
+# ------------------------------------------------------------------ grid + sampling
+@pytest.mark.parametrize("gt", [0, 1, 2])
+def test_grid_bitexact(tiny, oracle_mod, gt):
+    g, P, _ = tiny[gt]
+    d = g.export()
+    assert np.array_equal(d["E"], P.E)
+    assert np.array_equal(d["X"], P.X)
+    assert np.array_equal(d["mats"], P.mats)
+    assert np.array_equal(d["concs"], P.concs)
+    assert np.array_equal(d["num_nucs"], P.num_nucs)
+    if gt == 0:
+        assert np.array_equal(d["U"], P.U)
+        assert np.array_equal(d["IDX"], P.IDX)
+    if gt == 2:
+        assert np.array_equal(d["H"], P.H)
+
+
+def test_grid_small_bitexact_and_checksum(xs, oracle_mod):
+    w = WORKLOADS["small"]
+    g = xs.Grid(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    d = g.export()
+    assert np.array_equal(d["E"], P.E) and np.array_equal(d["X"], P.X) and np.array_equal(d["concs"], P.concs)
+    g2 = xs.Grid(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    assert g.checksum() == g2.checksum()
+    g3 = xs.Grid(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED + 1)
+    assert g3.checksum() != g.checksum()
+
+
+@pytest.mark.parametrize("first", [0, 12345, 2 ** 40 + 7, 2 ** 62 - 5000])
+def test_sample_bitexact(tiny, first):
+    g, P, _ = tiny[1]
+    n = 5000
+    q, m = g.sample(first, n, LOOKUP_SEED)
+    ref = P.run_range(LOOKUP_SEED, first, n, macro=False, mat=True, q=True)
+    assert np.array_equal(q.cpu().numpy(), ref["q"])
+    assert np.array_equal(m.cpu().numpy(), ref["mat"])
+
+
+# ------------------------------------------------------------------ tiny: full cross product
+@pytest.mark.parametrize("gt", [0, 1, 2])
+@pytest.mark.parametrize("search", SEARCHES)
+@pytest.mark.parametrize("sort", SORTS)
+def test_tiny_indices_bitexact(tiny, gt, search, sort):
+    g, P, ref = tiny[gt]
+    idx = g.indices(0, 100_000, LOOKUP_SEED, search=search, sort=sort)
+    assert np.array_equal(idx.cpu().numpy(), ref["idx"])
+
+
+@pytest.mark.parametrize("gt", [0, 1, 2])
+@pytest.mark.parametrize("search", SEARCHES)
+@pytest.mark.parametrize("sort", SORTS)
+def test_tiny_macro_and_hash(tiny, gt, search, sort):
+    g, P, ref = tiny[gt]
+    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, search=search, sort=sort)
+    assert st.hash == ref["hash"] and st.pairs == ref["pairs"] and st.lookups == 100_000
+    got = out.cpu().numpy()
+    assert _macro_close(got, ref["macro"]) <= RTOL
+    assert np.array_equal(got, ref["macro"])  # expected bit-exact (R8)
+
+
+# ------------------------------------------------------------------ edge cases
+@pytest.mark.parametrize("first,count", [(0, 0), (0, 1), (7, 31), (1000, 257), (99_000, 1000), (3, 4097)])
+@pytest.mark.parametrize("sort", SORTS)
+def test_ragged_ranges(tiny, first, count, sort):
+    g, P, ref = tiny[1]
+    out, st = g.macro_xs(first, count, LOOKUP_SEED, sort=sort)
+    r = P.run_range(LOOKUP_SEED, first, count)
+    assert st.hash == r["hash"] and st.pairs == r["pairs"]
+    assert np.array_equal(out.cpu().numpy(), r["macro"])
+
+
+@pytest.mark.parametrize("bins", [1, 2, 64, 1024, 4096])
+@pytest.mark.parametrize("block", [64, 128, 256])
+def test_energy_bins_and_block(tiny, bins, block):
+    g, P, ref = tiny[1]
+    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, sort="material_energy", energy_bins=bins, block=block)
+    assert st.hash == ref["hash"]
+    assert np.array_equal(out.cpu().numpy(), ref["macro"])
+
+
+def test_host_outputs(tiny, xs):
+    g, P, ref = tiny[1]
+    n = 100_000
+    pinned = torch.empty((n, 5), dtype=torch.float64).pin_memory()
+    st = g.lookup_range(0, n, LOOKUP_SEED, pinned)
+    assert st.hash == ref["hash"] and np.array_equal(pinned.numpy(), ref["macro"])
+    pageable = np.zeros((n, 5))
+    st = g.lookup_range(0, n, LOOKUP_SEED, pageable)
+    assert np.array_equal(pageable, ref["macro"])
+    assert xs.xs_lookup_batch(g.handle, n, LOOKUP_SEED, None) == ref["hash"]
+
+
+def test_invalid_opts(tiny, xs):
+    g, _, _ = tiny[1]
+    with pytest.raises(xs.XSError):
+        g.lookup_range(0, 10, LOOKUP_SEED, search=42)
+    with pytest.raises(xs.XSError):
+        g.lookup_range(0, 10, LOOKUP_SEED, energy_bins=3)
+    with pytest.raises(xs.XSError):
+        g.lookup_range(-1, 10, LOOKUP_SEED)
+    with pytest.raises(xs.XSError):
+        g.lookup_range(2 ** 62, 10, LOOKUP_SEED)
+
+
+@pytest.mark.parametrize("gt", [0, 1, 2])
+@pytest.mark.parametrize("search", SEARCHES)
+def test_search_points_edges(tiny, oracle_mod, gt, search):
+    """Arbitrary energies: every gridpoint, its neighbours, out of range, 0, 1, bin edges."""
+    g, P, _ = tiny[gt]
+    rng = np.random.default_rng(0)
+    nucs, qs = [], []
+    for nuc in (0, 17, 67):
+        E = P.E[nuc]
+        pts = np.concatenate([E, np.nextafter(E, -1), np.nextafter(E, 2), [-1.0, 0.0, 1.0, 2.0, E[0] / 2],
+                              np.arange(0, 10000, 13) / 10000.0, rng.random(500)])
+        qs.append(pts)
+        nucs.append(np.full(len(pts), nuc))
+    q = np.concatenate(qs)
+    nuc = np.concatenate(nucs).astype(np.int32)
+    L = g.search_points(q, nuc, search).cpu().numpy()
+    expect = np.array([oracle_mod.search_def(P.E[a], b) for a, b in zip(nuc, q)])
+    assert np.array_equal(L, expect)
+
+
+def test_determinism_and_shards(tiny):
+    g, P, ref = tiny[1]
+    hs = [g.lookup_range(0, 100_000, LOOKUP_SEED).hash for _ in range(3)]
+    assert hs == [ref["hash"]] * 3
+    cuts = [0, 12_345, 50_000, 77_777, 100_000]
+    assert sum(g.lookup_range(a, b - a, LOOKUP_SEED).hash for a, b in zip(cuts, cuts[1:])) == ref["hash"]
+
+
+# ------------------------------------------------------------------ full-size configs
+def _sampled_check(g, P, n_total, search="U2", sort="material_energy", n_samples=2000, prefix=200_000):
+    """Full-size launch (the bench configuration) on device, then sampled outputs + a prefix hash."""
+    out = torch.empty((n_total, 5), dtype=torch.float64, device=g.device)
+    st = g.lookup_range(0, n_total, LOOKUP_SEED, out, search=search, sort=sort)
+    rng = np.random.default_rng(1)
+    idx = np.unique(np.concatenate([rng.integers(0, n_total, n_samples), [0, n_total - 1]]))
+    _, ref_macro = P.run_indices(LOOKUP_SEED, idx)
+    got = out[torch.as_tensor(idx, device=g.device)].cpu().numpy()
+    assert _macro_close(got, ref_macro) <= RTOL
+    assert np.array_equal(got, ref_macro)
+    ref_prefix = P.run_range(LOOKUP_SEED, 0, prefix, macro=False)
+    assert g.lookup_range(0, prefix, LOOKUP_SEED, search=search, sort=sort).hash == ref_prefix["hash"]
+    # hash properties that hold at any size
+    assert st.lookups == n_total and n_total <= st.hash <= 5 * n_total
+    v = torch.argmax(out, dim=1)  # ties to the first maximum, like the kernel
+    assert int((v + 1).sum().item()) == st.hash
+    return st
+
+
+def test_small_full_hash(xs, oracle_mod):
+    w = WORKLOADS["small"]
+    g = xs.Grid(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    ref = P.run_range(LOOKUP_SEED, 0, w.lookups, macro=False)
+    for search in ("M", "U2", "U4"):
+        st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search=search)
+        assert st.hash == ref["hash"] and st.pairs == ref["pairs"]
+    st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search="U2", sort="none")
+    assert st.hash == ref["hash"]
+    _sampled_check(g, P, w.lookups)
+
+
+@pytest.mark.slow
+def test_large_nuclide_sampled(xs, oracle_mod):
+    w = WORKLOADS["large"]
+    g = xs.Grid(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
+    _sampled_check(g, P, w.lookups)
+    g.close()
+
+
+@pytest.mark.slow
+def test_large_unionized_sampled(xs, oracle_mod):
+    w = WORKLOADS["large-U"]
+    g = xs.Grid(w.n_nuclides, w.n_gridpoints, 0, GRID_SEED)
+    P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 0, GRID_SEED, build_idx=False)
+    # 100M x 40 B of output is 4 GB on device: fine on a B200
+    _sampled_check(g, P, w.lookups, n_samples=1000, prefix=100_000)
+    g.close()
+
+
+@pytest.mark.slow
+def test_xl_hash_sampled(xs, oracle_mod):
+    w = WORKLOADS["XL"]
+    g = xs.Grid(w.n_nuclides, w.n_gridpoints, 2, GRID_SEED)
+    P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 2, GRID_SEED)
+    n = 20_000_000  # a full-size range of the per-GPU XL share, sampled
+    _sampled_check(g, P, n, n_samples=1000, prefix=100_000)
+    st = g.lookup_range(0, w.lookups, LOOKUP_SEED)  # the bench launch: 125M lookups
+    assert st.lookups == w.lookups and w.lookups <= st.hash <= 5 * w.lookups
+    g.close()
