@@ -1,0 +1,315 @@
+#!/usr/bin/env python
+"""bench.py -- lookups/s of the XSBench-style macroscopic XS lookup on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload small] [--search U4] [--sort material_energy]
+
+One step = one pass of the whole hot path (sampling,
+(material, energy) ordering, search, interpolation, accumulation, verification) over
+one batch of lookups on every rank, inputs (the grid) resident in HBM.  Weak scaling:
+rank r owns lookups [r*L, (r+1)*L) of each batch (L = the workload's per-GPU count).
+Rank 0 prints ONE JSON line.  Timing: W untimed warm-up steps, then K steps, each
+bracketed by CUDA events on the launching stream with the 126 MB L2 flushed (a
+256 MiB write) before it, outside the events; barrier + synchronize on both sides;
+the max over ranks of the summed step times.  Grid creation is untimed (XSBench's
+grid_init_do_not_profile [XSB]).
+
+--impl reference times the CPU oracle (oracle/, plain C + OpenMP) on the box's host
+cores on a bounded sample of the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from xs_workloads import GRID_SEED, LOOKUP_SEED, MEAN_NUCS, WORKLOADS, GRID_NAMES  # noqa: E402
+
+METRIC = "lookups/sec (device-timed, max over ranks)"
+UNIT = "lookups/s"
+L2_FLUSH_BYTES = 256 << 20
+BYTES_PER_PAIR = 96  # two 48 B point records per (lookup, nuclide)
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--workload", default="small", choices=sorted(WORKLOADS))
+    p.add_argument("--lookups", type=int, default=0, help="override lookups per GPU")
+    p.add_argument("--search", default="U4")
+    p.add_argument("--sort", default="material_energy")
+    p.add_argument("--energy-bins", type=int, default=0)
+    p.add_argument("--no-flush", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=12.0, help="target wall time of the CPU sample")
+    return p.parse_args()
+
+
+def algorithmic_bytes_per_lookup(w) -> float:
+    """the useful bytes of a random gather -- E[n_nuc] x 96 B (nuclide),
+    + 4 B of IDX per pair (unionized), + 8*ceil(log2(W+1)) B of window probes (hash).
+    Probes into L2-resident search arrays are excluded."""
+    m = MEAN_NUCS[68 if w.n_nuclides == 68 else 355]
+    if w.grid_type == 1:
+        per_pair = BYTES_PER_PAIR
+    elif w.grid_type == 0:
+        per_pair = BYTES_PER_PAIR + 4
+    else:
+        W = w.n_gridpoints / 10000
+        per_pair = BYTES_PER_PAIR + 8 * math.ceil(math.log2(W + 1))
+    return m * per_pair
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(workload: str, search: str, sort: str):
+    """DRAM bytes per launch of k_lookup from the committed ncu --set full capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            d = json.load(f)
+        return d.get(f"{workload}/{search}/{sort}")
+    except Exception:
+        return None
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.p = None
+        self.path = os.path.join("/tmp", f"xs_clocks_{os.getpid()}.csv")
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+            time.sleep(0.3)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            try:
+                self.p.wait(timeout=5)
+            except Exception:
+                self.p.kill()
+            self.f.close()
+
+    def summary(self):
+        if not self.p:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        rows = []
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 9:
+                rows.append(parts)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = max(float(r[2]) for r in rows if r[2].replace(".", "").isdigit())
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in rows for k in range(4) if r[5 + k].lower() == "active"})
+        loaded = [s for s in sm if s > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def cpu_baseline(w, lookups_cap: int, seconds: float):
+    """The oracle as it stands on this host's cores: a bounded sample of the workload."""
+    import oracle
+    t0 = time.time()
+    P = oracle.Problem(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED, build_idx=False)
+    setup_s = time.time() - t0
+    threads = oracle.max_threads()
+    n = 20_000
+    t0 = time.perf_counter()
+    P.run_range(LOOKUP_SEED, 0, n, macro=False)
+    rate = n / max(time.perf_counter() - t0, 1e-6)
+    n = int(min(lookups_cap, max(n, rate * seconds)))
+    t0 = time.perf_counter()
+    r = P.run_range(LOOKUP_SEED, 0, n, macro=False)
+    dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"lookups [0, {n}) of {w.name} ({w.n_nuclides}x{w.n_gridpoints} "
+                      f"{GRID_NAMES[w.grid_type]}), OpenMP static over lookups, {dt:.1f} s wall "
+                      f"(grid build {setup_s:.1f} s untimed)",
+            "_hash": r["hash"], "_n": n}
+
+
+def run_reference(a, w):
+    """--impl reference: the oracle as the reference arm (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    P = oracle.Problem(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED, build_idx=False)
+    threads = oracle.max_threads()
+    n = 20_000
+    t0 = time.perf_counter()
+    P.run_range(LOOKUP_SEED, 0, n, macro=False)
+    rate = n / max(time.perf_counter() - t0, 1e-6)
+    budget = 150.0 / max(a.steps + a.warmup, 1)  # whole run within a few minutes
+    n = int(max(10_000, min(w.lookups, rate * budget)))
+    times = []
+    for k in range(a.warmup + a.steps):
+        t0 = time.perf_counter()
+        P.run_range(LOOKUP_SEED, 0, n, macro=False)
+        if k >= a.warmup:
+            times.append(time.perf_counter() - t0)
+    total = sum(times)
+    value = n * len(times) / total
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": a.gpus,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * total / len(times),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (XSBench LCG grid + lookups, seeds 42/1070)",
+        "config": {"workload": w.name, "n_nuclides": w.n_nuclides, "n_gridpoints": w.n_gridpoints,
+                   "grid": GRID_NAMES[w.grid_type], "lookups_per_step": n},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                         "sample": f"lookups [0, {n}) of {w.name} per step"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(a, w):
+    import torch
+    import paper_conf_cgo_murtovigplls24_b200 as xs
+    from paper_conf_cgo_murtovigplls24_b200 import driver
+
+    R = driver.init()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    L = a.lookups or w.lookups
+    first, count = driver.weak_range(L, R.rank)
+    g = xs.Grid(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED)
+    assert driver.replicas_identical(g.checksum()), "grid replicas differ across ranks"
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+    opts = dict(search=a.search, sort=a.sort, energy_bins=a.energy_bins, timing=True)
+
+    def step():
+        return g.lookup_range(first, count, LOOKUP_SEED, None, **opts)
+
+    ref_stats = None
+    for _ in range(a.warmup):
+        ref_stats = step()
+    driver.barrier()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    stats = []
+    with Clocks(torch.cuda.current_device()) as clk:
+        for k in range(a.steps):
+            if not a.no_flush:
+                flush.fill_(k)
+            ev[k][0].record(stream)
+            stats.append(step())
+            ev[k][1].record(stream)
+        torch.cuda.synchronize()
+    driver.barrier()
+    step_ms = [s.elapsed_time(e) for s, e in ev]
+    total_ms = driver.max_over_ranks(sum(step_ms))
+    lookup_ms = [s.lookup_ms for s in stats]
+    hashes = {s.hash for s in stats}
+    assert len(hashes) == 1 and (ref_stats is None or ref_stats.hash in hashes), "non-deterministic hash"
+    h, nl, npairs, _ = driver.reduce_stats(stats[0].hash, stats[0].lookups, stats[0].pairs, 0.0)
+
+    # ---- e2e: the public API with HOST output buffers (D2H of every macro XS in the region)
+    e2e = None
+    if not a.no_e2e:
+        host = torch.empty((count, 5), dtype=torch.float64).pin_memory()
+        for _ in range(2):
+            g.lookup_range(first, count, LOOKUP_SEED, host, search=a.search, sort=a.sort)
+        driver.barrier()
+        torch.cuda.synchronize()
+        t = []
+        for k in range(max(3, a.steps // 4)):
+            if not a.no_flush:
+                flush.fill_(k)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            g.lookup_range(first, count, LOOKUP_SEED, host, search=a.search, sort=a.sort)
+            t.append(time.perf_counter() - t0)
+        e2e_s = driver.max_over_ranks(sum(t))
+        e2e = {"value": R.world * count * len(t) / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 0,
+               "d2h_bytes_per_step": count * 5 * 8 + 16,
+               "note": "xs_lookup_range into pinned host memory, host wall clock; inputs are the "
+                       "(seed, range) scalars -- lookups are drawn on device by the method's "
+                       "counter-based LCG (DESIGN.md §8)"}
+
+    if R.rank != 0:
+        driver.finalize()
+        return
+    value = R.world * count * a.steps / (total_ms / 1e3)
+    peak, peak_src = measured_peaks()
+    bpl = algorithmic_bytes_per_lookup(w)
+    mean_lookup_ms = statistics.mean(lookup_ms)
+    achieved = bpl * count / (mean_lookup_ms / 1e3) / 1e9
+    traffic = ncu_traffic(w.name, a.search, a.sort)
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": R.world, "steps": a.steps,
+        "warmup": a.warmup, "ms_per_step": total_ms / a.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (XSBench LCG grid + lookups, seeds 42/1070)",
+        "config": {"workload": w.name, "n_nuclides": w.n_nuclides, "n_gridpoints": w.n_gridpoints,
+                   "grid": GRID_NAMES[w.grid_type], "lookups_per_gpu": count, "search": a.search,
+                   "sort": a.sort, "l2_flush": not a.no_flush, "parallelism": f"dp{R.world} (index ranges)"},
+        "step_ms": {"median": statistics.median(step_ms), "rsd_pct": 100 * statistics.pstdev(step_ms) /
+                    statistics.mean(step_ms), "min": min(step_ms), "max": max(step_ms)},
+        "phase_ms": {"sort": statistics.mean(s.sample_ms for s in stats), "lookup": mean_lookup_ms},
+        "roofline": {"bound": "hbm", "kernel": "k_lookup", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "bytes_per_lookup_alg": bpl, "peak_source": peak_src},
+        "verification": {"hash": h, "lookups": nl, "pairs": npairs},
+        "gpu_launches": int(sum(s.lookup_launches for s in stats)),
+        "e2e": e2e,
+    }
+    line["clocks"] = clk.summary()
+    if not a.no_cpu_baseline and R.world == 1:
+        cb = cpu_baseline(w, count, a.cpu_seconds)
+        # parity of the bench's own configuration on the oracle's sample range
+        gs = g.lookup_range(0, cb["_n"], LOOKUP_SEED, None, search=a.search, sort=a.sort)
+        line["verification"]["oracle_sample_hash_match"] = bool(gs.hash == cb["_hash"])
+        line["cpu_baseline"] = {k: v for k, v in cb.items() if not k.startswith("_")}
+    print(json.dumps(line), flush=True)
+    g.close()
+    driver.finalize()
+
+
+def main():
+    a = parse()
+    w = WORKLOADS[a.workload]
+    if a.impl == "reference":
+        run_reference(a, w)
+    else:
+        run_ours(a, w)
+
+
+if __name__ == "__main__":
+    main()

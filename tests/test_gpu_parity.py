@@ -194,8 +194,11 @@ def _sampled_check(g, P, n_total, search="U2", sort="material_energy", n_samples
     assert g.lookup_range(0, prefix, LOOKUP_SEED, search=search, sort=sort).hash == ref_prefix["hash"]
     # hash properties that hold at any size
     assert st.lookups == n_total and n_total <= st.hash <= 5 * n_total
-    v = torch.argmax(out, dim=1)  # ties to the first maximum, like the kernel
-    assert int((v + 1).sum().item()) == st.hash
+    # v = 1 + first argmax with XSBench's start value max = -1.0 (R10): prepend a -1.0
+    # column (extrapolated lookups, R6, can have every channel below -1.0)
+    aug = torch.cat([torch.full((n_total, 1), -1.0, dtype=out.dtype, device=out.device), out], dim=1)
+    v = torch.clamp(torch.argmax(aug, dim=1), min=1)
+    assert int(v.sum().item()) == st.hash
     return st
 
 
