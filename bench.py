@@ -287,7 +287,7 @@ def run_ours(a, w):
                      "frac": achieved / peak, "traffic": traffic,
                      "bytes_per_lookup_alg": bpl, "peak_source": peak_src},
         "verification": {"hash": h, "lookups": nl, "pairs": npairs},
-        "gpu_launches": int(sum(s.lookup_launches for s in stats)),
+        "gpu_launches": int(sum(s.launches for s in stats)),
         "e2e": e2e,
     }
     line["clocks"] = clk.summary()

@@ -70,7 +70,11 @@ enum {
 };
 
 /* Flags. */
-enum { XS_FLAG_TIMING = 1 }; /* fill the per-phase *_ms fields of xs_stats (CUDA events) */
+enum {
+    XS_FLAG_TIMING = 1, /* fill the per-phase *_ms fields of xs_stats (CUDA events)          */
+    XS_FLAG_SPLIT = 2   /* sorted modes: the split k_search -> k_interp pair instead of the one
+                           fused search+interpolation kernel (A/B of the two designs)          */
+};
 
 typedef struct xs_opts {
     int32_t search;      /* XS_SEARCH_*                                                 */
@@ -89,9 +93,10 @@ typedef struct xs_stats {
     uint64_t pairs;   /* sum of num_nucs[mat] = (lookup, nuclide) pairs interpolated         */
     double device_ms; /* CUDA-event time of the whole call on opts->stream                   */
     double sample_ms; /* XS_FLAG_TIMING: sampling + ordering kernels                          */
-    double lookup_ms; /* XS_FLAG_TIMING: the lookup kernel(s) alone                            */
+    double lookup_ms; /* XS_FLAG_TIMING: the lookup kernel(s): k_lookup, or k_search + k_interp */
+    double search_ms; /* XS_FLAG_TIMING: k_search alone (XS_FLAG_SPLIT; else 0)              */
     double copy_ms;   /* XS_FLAG_TIMING: device->host copy of out_macro_xs (host outputs)      */
-    int32_t lookup_launches; /* kernels launched by the call (all kinds)                      */
+    int32_t launches; /* CUDA kernels this call launched (all kinds)                          */
     int32_t reserved;
 } xs_stats;
 

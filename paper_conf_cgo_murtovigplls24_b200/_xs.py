@@ -12,7 +12,9 @@ import os
 import re
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libxs.so")
+# XS_LIB_VARIANT selects an experimental build (libxs_<variant>.so) for A/B probes only
+LIB_PATH = os.path.join(_HERE, "libxs.so" if not os.environ.get("XS_LIB_VARIANT")
+                        else f"libxs_{os.environ['XS_LIB_VARIANT']}.so")
 HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "xs.h")
 
 if not os.path.exists(LIB_PATH):
@@ -29,6 +31,7 @@ XS_OK, XS_EINVAL, XS_ENOMEM, XS_ECUDA, XS_EDUP = 0, -1, -2, -3, -4
 XS_SEARCH_COUNT = 9
 XS_SORT_NONE, XS_SORT_MATERIAL, XS_SORT_MATERIAL_ENERGY = 0, 1, 2
 XS_FLAG_TIMING = 1
+XS_FLAG_SPLIT = 2
 
 SEARCH_NAMES = {"M": 0, "U1": 1, "U2": 2, "U4": 3, "U8": 4, "B": 5, "M2": 6, "M4": 7, "M8": 8}
 SORT_NAMES = {"none": 0, "material": 1, "material_energy": 2}
@@ -43,7 +46,8 @@ class xs_opts(C.Structure):
 class xs_stats(C.Structure):
     _fields_ = [("hash", C.c_uint64), ("lookups", C.c_uint64), ("pairs", C.c_uint64),
                 ("device_ms", C.c_double), ("sample_ms", C.c_double), ("lookup_ms", C.c_double),
-                ("copy_ms", C.c_double), ("lookup_launches", C.c_int32), ("reserved", C.c_int32)]
+                ("search_ms", C.c_double), ("copy_ms", C.c_double), ("launches", C.c_int32),
+                ("reserved", C.c_int32)]
 
 
 class xs_grid_info(C.Structure):

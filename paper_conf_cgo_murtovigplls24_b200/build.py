@@ -14,8 +14,8 @@ LIB = os.path.join(HERE, "libxs.so")
 BUILD = os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
-SOURCES = ["api.cu", "grid.cu", "lookup.cu"]
-HEADERS = ["rng.cuh", "search.cuh", "xs_internal.cuh"]
+SOURCES = ["api.cu", "grid.cu", "sort.cu", "lookup_fused.cu", "lookup_split.cu", "pipeline.cu"]
+HEADERS = ["rng.cuh", "search.cuh", "xs_internal.cuh", "lookup_common.cuh"]
 FLAGS = [
     "-O3", "-std=c++17",
     "-gencode", "arch=compute_100a,code=sm_100a",
@@ -35,10 +35,10 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def _compile(src: str) -> str:
-    obj = os.path.join(BUILD, src.replace(".cu", ".o"))
-    log = os.path.join(BUILD, src.replace(".cu", ".ptxas.log"))
-    cmd = [NVCC, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
+def _compile(src: str, bdir: str = BUILD, defines=()) -> str:
+    obj = os.path.join(bdir, src.replace(".cu", ".o"))
+    log = os.path.join(bdir, src.replace(".cu", ".ptxas.log"))
+    cmd = [NVCC, *FLAGS, *defines, "-c", os.path.join(CSRC, src), "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     with open(log, "w") as f:
         f.write(r.stdout + r.stderr)
@@ -47,20 +47,26 @@ def _compile(src: str) -> str:
     return obj
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """defines/out: experimental variants (e.g. -DXS_LOOKUP_MIN_BLOCKS=4 into libxs_mb4.so);
+    the product is always libxs.so built with no extra defines."""
+    lib = out or LIB
+    if not force and not defines and out is None and not _stale():
         return LIB
-    os.makedirs(BUILD, exist_ok=True)
+    bdir = BUILD if not defines else BUILD + "_" + "_".join(d.strip("-D").replace("=", "") for d in defines)
+    os.makedirs(bdir, exist_ok=True)
     with cf.ThreadPoolExecutor(len(SOURCES)) as ex:
-        objs = list(ex.map(_compile, SOURCES))
-    tmp = LIB + ".tmp"
+        objs = list(ex.map(lambda s: _compile(s, bdir, defines), SOURCES))
+    tmp = lib + ".tmp"
     cmd = [NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", tmp, *objs]
     subprocess.run(cmd, check=True)
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     if verbose:
         print(f"built {LIB}", file=sys.stderr)
     return LIB
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose=True)
+    defs = tuple(a for a in sys.argv[1:] if a.startswith("-D"))
+    outs = [a.split("=", 1)[1] for a in sys.argv[1:] if a.startswith("--out=")]
+    build(force="--force" in sys.argv, verbose=True, defines=defs, out=outs[0] if outs else None)

@@ -279,6 +279,11 @@ void free_grid(Grid &g)
         cudaFreeHost(g.stats_h);
     cudaFree(g.sq);
     cudaFree(g.si);
+    cudaFree(g.skey);
+    cudaFree(g.qs);
+    cudaFree(g.Lbuf);
+    if (g.mb_h)
+        cudaFreeHost(g.mb_h);
     cudaFree(g.hist);
     cudaFree(g.base);
     cudaFree(g.stage);

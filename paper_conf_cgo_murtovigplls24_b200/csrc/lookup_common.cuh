@@ -1,0 +1,150 @@
+// lookup_common.cuh -- device pieces shared by the lookup kernels.
+#pragma once
+#include "search.cuh"
+#include "xs_internal.cuh"
+
+namespace xs {
+
+// ---- sampling ------------------------------------------------
+// `s` is skip(seed, 2i): q is the draw at stream position 2i, the pick_mat roll at 2i+1.
+__device__ __forceinline__ void sample_lookup(uint64_t s, const SampleView &sv, double &q, int &mat)
+{
+    uint64_t t = lcg_step(s);
+    q = u63_to_double(t);
+    t = lcg_step(t);
+    const double roll = u63_to_double(t);
+    // pick_mat (R9): the first m in 1..11 with roll < T[m], else 0 (T is increasing)
+    int m = 0;
+#pragma unroll
+    for (int k = 11; k >= 1; k--)
+        m = (roll < sv.T[k]) ? k : m;
+    mat = m;
+}
+
+// skip(seed, 2*(first + j)) with the Listing-7 loop (kept merged: PAPER.md:474)
+__device__ __forceinline__ uint64_t lookup_state(const SampleView &sv, int64_t j)
+{
+    return lcg_apply(lcg_jump(2 * (uint64_t)(sv.first + j)), sv.seed);
+}
+
+__device__ __forceinline__ int energy_bucket(double q, int nb_log2)
+{
+    const int nb = 1 << nb_log2;
+    const int b = (int)__dmul_rn(q, (double)nb); // exact: nb is a power of two
+    return b < nb - 1 ? b : nb - 1;              // q may be exactly 1.0 (R7)
+}
+
+// material of sorted position j: the number of later materials whose first slot is <= j
+__device__ __forceinline__ int material_of(const uint32_t *mb, uint32_t j)
+{
+    int mat = 0;
+#pragma unroll
+    for (int m = 1; m < kMaterials; m++)
+        mat += (j >= mb[m]) ? 1 : 0;
+    return mat;
+}
+
+// ---- the lower index of one (lookup, nuclide) pair ----------------------
+template <int GRID, int SEARCH>
+__device__ __forceinline__ int lower_index(const GridView &gv, const double *__restrict__ Ei, int nuc, double q,
+                                           int e_union)
+{
+    if constexpr (GRID == XS_NUCLIDE) {
+        return search<SEARCH>(Ei, 0, gv.n - 1, q);
+    } else if constexpr (GRID == XS_UNIONIZED) {
+        return __ldg(gv.IDX + (size_t)e_union * (uint32_t)gv.n_nuc + nuc);
+    } else { // hash window with guards (R7)
+        int64_t b = (int64_t)__ddiv_rn(q, gv.du);
+        b = b < 0 ? 0 : (b > gv.bins - 1 ? gv.bins - 1 : b);
+        const int lo = __ldg(gv.H + b * gv.n_nuc + nuc);
+        const int hi = (b == gv.bins - 1) ? gv.n - 1 : __ldg(gv.H + (b + 1) * gv.n_nuc + nuc) + 1;
+        if (q < __ldg(Ei + lo) || (hi < gv.n - 1 && q >= __ldg(Ei + hi)))
+            return search<SEARCH>(Ei, 0, gv.n - 1, q);
+        return search<SEARCH>(Ei, lo, hi, q);
+    }
+}
+
+template <int GRID, int SEARCH>
+__device__ __forceinline__ int union_index(const GridView &gv, double q)
+{
+    if constexpr (GRID == XS_UNIONIZED)
+        return search<SEARCH>(opaque(gv.U), 0, gv.N - 1, q);
+    else
+        return 0;
+}
+
+__device__ __forceinline__ const double *nuclide_row(const GridView &gv, int nuc)
+{
+    return opaque(gv.E + (size_t)nuc * (uint32_t)gv.n);
+}
+
+// ---- interpolation + accumulation of one pair (reading R8) ------------------------------
+struct Acc {
+    double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0, a4 = 0.0;
+};
+
+// 96 B gather: the 48 B records of points L and L+1, three 16 B loads each
+__device__ __forceinline__ void accumulate_pair(const GridView &gv, int nuc, int L, double q, double conc, Acc &A)
+{
+    const double2 *p = reinterpret_cast<const double2 *>(gv.pts) + ((size_t)nuc * (uint32_t)gv.n + L) * 3;
+    const double2 l0 = __ldg(p + 0), l1 = __ldg(p + 1), l2 = __ldg(p + 2);
+    const double2 h0 = __ldg(p + 3), h1 = __ldg(p + 4), h2 = __ldg(p + 5);
+    const double f = __ddiv_rn(__dsub_rn(h0.x, q), __dsub_rn(h0.x, l0.x));
+    A.a0 = __fma_rn(__fma_rn(-f, __dsub_rn(h0.y, l0.y), h0.y), conc, A.a0);
+    A.a1 = __fma_rn(__fma_rn(-f, __dsub_rn(h1.x, l1.x), h1.x), conc, A.a1);
+    A.a2 = __fma_rn(__fma_rn(-f, __dsub_rn(h1.y, l1.y), h1.y), conc, A.a2);
+    A.a3 = __fma_rn(__fma_rn(-f, __dsub_rn(h2.x, l2.x), h2.x), conc, A.a3);
+    A.a4 = __fma_rn(__fma_rn(-f, __dsub_rn(h2.y, l2.y), h2.y), conc, A.a4);
+}
+
+// verification value (R10): 1 + first maximum, strict '>' from -1.0
+__device__ __forceinline__ uint32_t verify(const Acc &A)
+{
+    double mx = -1.0;
+    uint32_t v = 0;
+    if (A.a0 > mx) { mx = A.a0; v = 0; }
+    if (A.a1 > mx) { mx = A.a1; v = 1; }
+    if (A.a2 > mx) { mx = A.a2; v = 2; }
+    if (A.a3 > mx) { mx = A.a3; v = 3; }
+    if (A.a4 > mx) { mx = A.a4; v = 4; }
+    return v + 1;
+}
+
+__device__ __forceinline__ void store_macro(double *__restrict__ out, uint32_t r, const Acc &A)
+{
+    double *o = out + (size_t)r * 5;
+    o[0] = A.a0;
+    o[1] = A.a1;
+    o[2] = A.a2;
+    o[3] = A.a3;
+    o[4] = A.a4;
+}
+
+// fused epilogue: CTA reduction of (hash, pairs), one 64-bit atomic per counter per CTA
+template <int TPB>
+__device__ __forceinline__ void reduce_stats(uint32_t my_hash, uint32_t my_pairs, unsigned long long *stats)
+{
+    __shared__ uint32_t s_red[2][TPB / 32];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        my_hash += __shfl_down_sync(0xffffffffu, my_hash, o);
+        my_pairs += __shfl_down_sync(0xffffffffu, my_pairs, o);
+    }
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (lane == 0) {
+        s_red[0][wid] = my_hash;
+        s_red[1][wid] = my_pairs;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long h = 0, pr = 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) {
+            h += s_red[0][w];
+            pr += s_red[1][w];
+        }
+        atomicAdd(stats + 0, h);
+        atomicAdd(stats + 1, pr);
+    }
+}
+
+} // namespace xs

@@ -1,0 +1,222 @@
+// sort.cu -- sampling + the (material, energy) counting sort.
+//
+// Key = (material << nb_log2) | energy bucket, K = 12 << nb_log2 <= 49152 buckets.
+//   k_bucket_count   sample each lookup of the chunk once (one Listing-7 jump per thread,
+//                    then one affine step per lookup), write its energy and key at its own
+//                    offset (coalesced) and histogram the keys in shared memory
+//   k_bucket_colscan per bucket, exclusive scan over CTAs (loads batched by 8)
+//   k_bucket_base    exclusive scan of the bucket totals + material bases (one CTA)
+//   k_bucket_scatter scatter the 4 B lookup offsets to their slots: 68 MB for 17M lookups,
+//                    L2-resident, so the random partial-sector writes merge in L2
+//   k_bucket_gather  (split path only) q in slot order; the fused lookup kernel instead
+//                    prefetches q_of[slot] one grid-stride iteration ahead
+// Order inside a bucket is whatever the shared-memory atomics give; results never depend
+// on it (every lookup is independent and the hash is an integer sum).
+#include <algorithm>
+
+#include "lookup_common.cuh"
+
+namespace xs {
+
+constexpr int kSortTpb = 1024;
+
+__global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, int nb_log2, int per_cta, Affine J_tpb,
+                                                            uint32_t *__restrict__ hist, double *__restrict__ q_of,
+                                                            uint16_t *__restrict__ key_of)
+{
+    extern __shared__ uint32_t sh[];
+    const int K = kMaterials << nb_log2;
+    for (int k = threadIdx.x; k < K; k += kSortTpb)
+        sh[k] = 0;
+    __syncthreads();
+    const int count = (int)sv.count;
+    const int beg = blockIdx.x * per_cta;
+    const int end = min(beg + per_cta, count);
+    int j = beg + threadIdx.x;
+    if (j < end) {
+        uint64_t s = lookup_state(sv, j);
+        for (; j < end; j += kSortTpb) {
+            double q;
+            int mat;
+            sample_lookup(s, sv, q, mat);
+            const int key = (mat << nb_log2) + energy_bucket(q, nb_log2);
+            atomicAdd(&sh[key], 1u);
+            q_of[j] = q;
+            key_of[j] = (uint16_t)key;
+            s = lcg_apply(J_tpb, s);
+        }
+    }
+    __syncthreads();
+    uint32_t *h = hist + (int64_t)blockIdx.x * K;
+    for (int k = threadIdx.x; k < K; k += kSortTpb)
+        h[k] = sh[k];
+}
+
+__global__ void k_bucket_colscan(int K, int ctas, uint32_t *hist, uint32_t *__restrict__ total)
+{
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= K)
+        return;
+    uint32_t run = 0;
+    int c = 0;
+    for (; c + 8 <= ctas; c += 8) {
+        uint32_t v[8];
+#pragma unroll
+        for (int u = 0; u < 8; u++)
+            v[u] = hist[(int64_t)(c + u) * K + k];
+#pragma unroll
+        for (int u = 0; u < 8; u++) {
+            hist[(int64_t)(c + u) * K + k] = run;
+            run += v[u];
+        }
+    }
+    for (; c < ctas; c++) {
+        const uint32_t v = hist[(int64_t)c * K + k];
+        hist[(int64_t)c * K + k] = run;
+        run += v;
+    }
+    total[k] = run;
+}
+
+__global__ void __launch_bounds__(1024) k_bucket_base(int K, int nb_log2, uint32_t *__restrict__ base)
+{
+    __shared__ uint32_t wsum[32];
+    __shared__ uint32_t carry;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (threadIdx.x == 0)
+        carry = 0;
+    __syncthreads();
+    for (int r0 = 0; r0 < K; r0 += 1024) {
+        const int k = r0 + threadIdx.x;
+        const uint32_t v = k < K ? base[k] : 0u;
+        uint32_t incl = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o)
+                incl += t;
+        }
+        if (lane == 31)
+            wsum[wid] = incl;
+        __syncthreads();
+        if (wid == 0) {
+            uint32_t w = wsum[lane];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t t = __shfl_up_sync(0xffffffffu, w, o);
+                if (lane >= o)
+                    w += t;
+            }
+            wsum[lane] = w;
+        }
+        __syncthreads();
+        const uint32_t c0 = carry;
+        if (k < K)
+            base[k] = c0 + incl - v + (wid ? wsum[wid - 1] : 0u);
+        __syncthreads();
+        if (threadIdx.x == 0)
+            carry = c0 + wsum[31];
+        __syncthreads();
+    }
+    if (threadIdx.x < kMaterials)
+        base[K + threadIdx.x] = base[threadIdx.x << nb_log2];
+    if (threadIdx.x == 0)
+        base[K + kMaterials] = carry;
+}
+
+__global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int nb_log2, int per_cta, int count,
+                                                              const uint32_t *__restrict__ hist,
+                                                              const uint32_t *__restrict__ base,
+                                                              const uint16_t *__restrict__ key_of,
+                                                              uint32_t *__restrict__ slot_of)
+{
+    extern __shared__ uint32_t sh[];
+    const int K = kMaterials << nb_log2;
+    const uint32_t *h = hist + (int64_t)blockIdx.x * K;
+    for (int k = threadIdx.x; k < K; k += kSortTpb)
+        sh[k] = base[k] + h[k];
+    __syncthreads();
+    const int beg = blockIdx.x * per_cta;
+    const int end = min(beg + per_cta, count);
+    for (int j = beg + threadIdx.x; j < end; j += kSortTpb) {
+        const uint32_t pos = atomicAdd(&sh[key_of[j]], 1u);
+        slot_of[pos] = (uint32_t)j;
+    }
+}
+
+__global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of, const double *__restrict__ q_of,
+                                double *__restrict__ q_sorted)
+{
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < count; j += gridDim.x * blockDim.x)
+        q_sorted[j] = __ldg(q_of + __ldg(slot_of + j));
+}
+
+static int sm_count_dev()
+{
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return sms > 0 ? sms : 148;
+}
+
+static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
+{
+    if (g.cap < chunk) {
+        cudaFree(g.sq);
+        cudaFree(g.si);
+        cudaFree(g.skey);
+        cudaFree(g.qs);
+        g.sq = g.qs = nullptr;
+        g.si = nullptr;
+        g.skey = nullptr;
+        g.cap = 0;
+        XS_CUDA_TRY(cudaMalloc(&g.sq, (size_t)chunk * sizeof(double)));
+        XS_CUDA_TRY(cudaMalloc(&g.qs, (size_t)chunk * sizeof(double)));
+        XS_CUDA_TRY(cudaMalloc(&g.si, (size_t)chunk * sizeof(uint32_t)));
+        XS_CUDA_TRY(cudaMalloc(&g.skey, (size_t)chunk * sizeof(uint16_t)));
+        g.cap = chunk;
+    }
+    const int64_t need = (int64_t)ctas * K;
+    if (g.hist_cap < need) {
+        cudaFree(g.hist);
+        cudaFree(g.base);
+        g.hist = nullptr;
+        g.base = nullptr;
+        g.hist_cap = 0;
+        XS_CUDA_TRY(cudaMalloc(&g.hist, (size_t)need * sizeof(uint32_t)));
+        XS_CUDA_TRY(cudaMalloc(&g.base, (size_t)(kMaterials * kMaxEnergyBins + 32) * sizeof(uint32_t)));
+        g.hist_cap = need;
+    }
+}
+
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gather, cudaStream_t stream)
+{
+    static bool smem_set[64] = {};
+    if (!smem_set[g.device & 63]) {
+        const int bytes = kMaterials * kMaxEnergyBins * 4;
+        XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_count, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+        XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+        smem_set[g.device & 63] = true;
+    }
+    const int64_t cn = sv.count;
+    const int K = kMaterials << nb_log2;
+    const int sms = sm_count_dev();
+    const int ctas = (int)std::max<int64_t>(1, std::min<int64_t>(sms, (cn + kSortTpb - 1) / kSortTpb));
+    const int per_cta = (int)((cn + ctas - 1) / ctas);
+    ensure_sort_space(g, cn, ctas, K);
+    const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
+    const size_t smem = (size_t)K * 4;
+    k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, nb_log2, per_cta, J, g.hist, g.sq, g.skey);
+    k_bucket_colscan<<<(K + 127) / 128, 128, 0, stream>>>(K, ctas, g.hist, g.base);
+    k_bucket_base<<<1, 1024, 0, stream>>>(K, nb_log2, g.base);
+    k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(nb_log2, per_cta, (int)cn, g.hist, g.base, g.skey, g.si);
+    XS_CUDA_TRY(cudaGetLastError());
+    if (!with_gather)
+        return 4;
+    const int gblocks = (int)std::min<int64_t>((cn + 255) / 256, (int64_t)sms * 8);
+    k_bucket_gather<<<gblocks, 256, 0, stream>>>((int)cn, g.si, g.sq, g.qs);
+    XS_CUDA_TRY(cudaGetLastError());
+    return 5;
+}
+
+} // namespace xs

@@ -64,8 +64,13 @@ struct Grid {
     // per-grid scratch (grown on demand; calls on one grid are serialised by the caller)
     uint64_t *stats_d = nullptr;     // [4] hash, pairs
     uint64_t *stats_h = nullptr;     // pinned mirror
-    double *sq = nullptr;            // sorted energies       [cap]
-    uint32_t *si = nullptr;          // sorted lookup offsets [cap]
+    double *sq = nullptr;            // energies by lookup offset (coalesced writes) [cap]
+    uint32_t *si = nullptr;          // lookup offsets in (material, energy) order  [cap]
+    uint16_t *skey = nullptr;        // bucket key by lookup offset                [cap]
+    double *qs = nullptr;            // energies in (material, energy) order       [cap]
+    int32_t *Lbuf = nullptr;         // split path: lower index of every pair      [lcap]
+    int64_t lcap = 0;
+    uint32_t *mb_h = nullptr;        // pinned: material bases of the last sort
     uint32_t *hist = nullptr;        // per-CTA bucket histograms [ctas][K]
     uint32_t *base = nullptr;        // [K + 16]: bucket bases, then material bases
     int64_t cap = 0, hist_cap = 0;
@@ -118,12 +123,47 @@ struct SampleView {
 GridView make_view(const Grid &g);
 SampleView make_sample_view(const Grid &g, uint64_t seed, int64_t first, int64_t count);
 
+// Lookups of one chunk in (material, energy) order.
+struct SortedView {
+    const double *__restrict__ q;        // split path: energy of sorted slot j (gathered)
+    const double *__restrict__ q_of;     // energy by lookup offset
+    const uint32_t *__restrict__ slot;   // lookup offset (i - first) of sorted slot j
+    const uint32_t *__restrict__ mb_dev; // device copy of matbase (fused path)
+    uint32_t matbase[kMaterials + 1];    // split path: first slot of each material; [12] = count
+};
+
+// Pair buffer of the split path: material m's pairs start at pairbase[m], laid out
+// nuclide-major ([jn][j - matbase[m]]) so a warp's stores and loads coalesce.
+struct PairView {
+    int32_t *__restrict__ L;
+    uint64_t pairbase[kMaterials];
+};
+
 // grid.cu
 void build_grid(Grid &g);
 void free_grid(Grid &g);
 uint64_t grid_checksum(const Grid &g);
 
-// lookup.cu
+// sort.cu: the (material, energy) counting sort of one chunk; leaves g.sq (energy by
+// lookup offset) and g.si (slot -> offset) filled and the material bases at g.base + K
+// (device).  with_gather also fills g.qs (energy by slot).  Returns kernels launched.
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gather, cudaStream_t stream);
+
+// lookup_fused.cu: one kernel per lookup batch (search + interpolation in one thread)
+void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, cudaStream_t stream,
+                  const GridView &gv, const SampleView &sv, const SortedView &so, Affine J_grid, double *out,
+                  int32_t *out_idx, unsigned long long *stats);
+
+// lookup_split.cu: k_search (every pair's lower index into the pair buffer; the paper's
+// loop, alone, at full occupancy) then k_interp (gather + interpolate + accumulate)
+void launch_search(int grid_type, int search, int blocks, cudaStream_t stream, const GridView &gv,
+                   const SortedView &so, const PairView &pv);
+void launch_interp(int blocks, cudaStream_t stream, const GridView &gv, const SortedView &so, const PairView &pv,
+                   double *out, int32_t *out_idx, unsigned long long *stats);
+constexpr int kSearchTpb = 256;
+constexpr int kInterpTpb = 256;
+
+// pipeline.cu
 void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
                  int32_t *out_idx, xs_stats *st);
 void run_sample(Grid &g, int64_t first, int64_t count, uint64_t seed, double *q, int32_t *mat, cudaStream_t s);

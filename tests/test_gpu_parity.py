@@ -86,21 +86,26 @@ def test_sample_bitexact(tiny, first):
 
 
 # ------------------------------------------------------------------ tiny: full cross product
+# (sort, split): the XSBench order; sorted + the fused kernel; sorted + k_search/k_interp
+PIPES = [("none", False), ("material", False), ("material_energy", False), ("material", True),
+         ("material_energy", True)]
+
+
 @pytest.mark.parametrize("gt", [0, 1, 2])
 @pytest.mark.parametrize("search", SEARCHES)
-@pytest.mark.parametrize("sort", SORTS)
-def test_tiny_indices_bitexact(tiny, gt, search, sort):
+@pytest.mark.parametrize("sort,split", PIPES)
+def test_tiny_indices_bitexact(tiny, gt, search, sort, split):
     g, P, ref = tiny[gt]
-    idx = g.indices(0, 100_000, LOOKUP_SEED, search=search, sort=sort)
+    idx = g.indices(0, 100_000, LOOKUP_SEED, search=search, sort=sort, split=split)
     assert np.array_equal(idx.cpu().numpy(), ref["idx"])
 
 
 @pytest.mark.parametrize("gt", [0, 1, 2])
 @pytest.mark.parametrize("search", SEARCHES)
-@pytest.mark.parametrize("sort", SORTS)
-def test_tiny_macro_and_hash(tiny, gt, search, sort):
+@pytest.mark.parametrize("sort,split", PIPES)
+def test_tiny_macro_and_hash(tiny, gt, search, sort, split):
     g, P, ref = tiny[gt]
-    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, search=search, sort=sort)
+    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, search=search, sort=sort, split=split)
     assert st.hash == ref["hash"] and st.pairs == ref["pairs"] and st.lookups == 100_000
     got = out.cpu().numpy()
     assert _macro_close(got, ref["macro"]) <= RTOL
@@ -109,10 +114,10 @@ def test_tiny_macro_and_hash(tiny, gt, search, sort):
 
 # ------------------------------------------------------------------ edge cases
 @pytest.mark.parametrize("first,count", [(0, 0), (0, 1), (7, 31), (1000, 257), (99_000, 1000), (3, 4097)])
-@pytest.mark.parametrize("sort", SORTS)
-def test_ragged_ranges(tiny, first, count, sort):
+@pytest.mark.parametrize("sort,split", PIPES)
+def test_ragged_ranges(tiny, first, count, sort, split):
     g, P, ref = tiny[1]
-    out, st = g.macro_xs(first, count, LOOKUP_SEED, sort=sort)
+    out, st = g.macro_xs(first, count, LOOKUP_SEED, sort=sort, split=split)
     r = P.run_range(LOOKUP_SEED, first, count)
     assert st.hash == r["hash"] and st.pairs == r["pairs"]
     assert np.array_equal(out.cpu().numpy(), r["macro"])
@@ -208,8 +213,9 @@ def test_small_full_hash(xs, oracle_mod):
     P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
     ref = P.run_range(LOOKUP_SEED, 0, w.lookups, macro=False)
     for search in ("M", "U2", "U4"):
-        st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search=search)
-        assert st.hash == ref["hash"] and st.pairs == ref["pairs"]
+        for split in (False, True):
+            st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search=search, split=split)
+            assert st.hash == ref["hash"] and st.pairs == ref["pairs"]
     st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search="U2", sort="none")
     assert st.hash == ref["hash"]
     _sampled_check(g, P, w.lookups)
