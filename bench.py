@@ -47,12 +47,14 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="small", choices=sorted(WORKLOADS))
     p.add_argument("--lookups", type=int, default=0, help="override lookups per GPU")
-    p.add_argument("--search", default="U4")
+    p.add_argument("--search", default="W")
     p.add_argument("--sort", default="material_energy")
     p.add_argument("--energy-bins", type=int, default=0)
     p.add_argument("--no-flush", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--ab", default="M,U1,U2,U4,U8,B,W", help="search variants for the A/B sub-object ('' = off)")
+    p.add_argument("--ab-steps", type=int, default=5)
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target wall time of the CPU sample")
     return p.parse_args()
 
@@ -81,8 +83,9 @@ def measured_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic(workload: str, search: str, sort: str):
-    """DRAM bytes per launch of k_lookup from the committed ncu --set full capture."""
+def ncu_record(workload: str, search: str, sort: str):
+    """The committed ncu --set full capture of k_lookup for this configuration
+    (profiles/ncu_traffic.json: DRAM bytes and warp instructions per launch)."""
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
             d = json.load(f)
@@ -214,31 +217,52 @@ def run_ours(a, w):
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
     opts = dict(search=a.search, sort=a.sort, energy_bins=a.energy_bins, timing=True)
 
-    def step():
-        return g.lookup_range(first, count, LOOKUP_SEED, None, **opts)
+    def step(**o):
+        return g.lookup_range(first, count, LOOKUP_SEED, None, **{**opts, **o})
+
+    def timed_steps(k_steps, **o):
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(k_steps)]
+        out = []
+        for k in range(k_steps):
+            if not a.no_flush:
+                flush.fill_(k)
+            evs[k][0].record(stream)
+            out.append(step(**o))
+            evs[k][1].record(stream)
+        torch.cuda.synchronize()
+        return [s_.elapsed_time(e_) for s_, e_ in evs], out
 
     ref_stats = None
     for _ in range(a.warmup):
         ref_stats = step()
     driver.barrier()
     torch.cuda.synchronize()
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
-    stats = []
     with Clocks(torch.cuda.current_device()) as clk:
-        for k in range(a.steps):
-            if not a.no_flush:
-                flush.fill_(k)
-            ev[k][0].record(stream)
-            stats.append(step())
-            ev[k][1].record(stream)
-        torch.cuda.synchronize()
+        step_ms, stats = timed_steps(a.steps)
     driver.barrier()
-    step_ms = [s.elapsed_time(e) for s, e in ev]
     total_ms = driver.max_over_ranks(sum(step_ms))
     lookup_ms = [s.lookup_ms for s in stats]
     hashes = {s.hash for s in stats}
     assert len(hashes) == 1 and (ref_stats is None or ref_stats.hash in hashes), "non-deterministic hash"
     h, nl, npairs, _ = driver.reduce_stats(stats[0].hash, stats[0].lookups, stats[0].pairs, 0.0)
+
+    # ---- the paper's A/B on this workload: every search variant, same protocol, fewer steps
+    ab = {}
+    for v in [x for x in a.ab.split(",") if x]:
+        for _ in range(2):
+            step(search=v)
+        ms, sts = timed_steps(a.ab_steps, search=v)
+        ms_max = driver.max_over_ranks(sum(ms))
+        ab[v] = {"value": R.world * count * a.ab_steps / (ms_max / 1e3),
+                 "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
+    if a.ab:
+        for _ in range(2):
+            step(search="M", sort="none")
+        ms, sts = timed_steps(a.ab_steps, search="M", sort="none")
+        ms_max = driver.max_over_ranks(sum(ms))
+        ab["M/unsorted (XSBench order)"] = {"value": R.world * count * a.ab_steps / (ms_max / 1e3),
+                                            "lookup_ms": statistics.mean(x.lookup_ms for x in sts),
+                                            "hash_ok": all(x.hash == stats[0].hash for x in sts)}
 
     # ---- e2e: the public API with HOST output buffers (D2H of every macro XS in the region)
     e2e = None
@@ -271,7 +295,8 @@ def run_ours(a, w):
     bpl = algorithmic_bytes_per_lookup(w)
     mean_lookup_ms = statistics.mean(lookup_ms)
     achieved = bpl * count / (mean_lookup_ms / 1e3) / 1e9
-    traffic = ncu_traffic(w.name, a.search, a.sort)
+    rec = ncu_record(w.name, a.search, a.sort)
+    traffic = rec["dram_bytes_per_launch"] if rec else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": R.world, "steps": a.steps,
         "warmup": a.warmup, "ms_per_step": total_ms / a.steps, "higher_is_better": True,
@@ -285,12 +310,23 @@ def run_ours(a, w):
         "phase_ms": {"sort": statistics.mean(s.sample_ms for s in stats), "lookup": mean_lookup_ms},
         "roofline": {"bound": "hbm", "kernel": "k_lookup", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
-                     "bytes_per_lookup_alg": bpl, "peak_source": peak_src},
+                     "bytes_per_lookup_alg": bpl, "peak_source": peak_src,
+                     "note": "achieved = SURVEY.md §8d random-gather bytes (E[nuclides] x 96 B per lookup) / "
+                             "k_lookup event time.  The (material, energy) sort makes warps share grid "
+                             "points, so DRAM traffic (`traffic`, ncu) is far below the algorithmic bytes "
+                             "and frac can exceed 1; the kernel is latency-bound (DESIGN.md §7)"},
+        "ab": ab,
         "verification": {"hash": h, "lookups": nl, "pairs": npairs},
         "gpu_launches": int(sum(s.launches for s in stats)),
         "e2e": e2e,
     }
     line["clocks"] = clk.summary()
+    if rec and rec.get("warp_inst_per_launch") and line["clocks"].get("sm_mhz"):
+        sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        ips = rec["warp_inst_per_launch"] / (mean_lookup_ms / 1e3)
+        peak_ips = sms * 4 * line["clocks"]["sm_mhz"] * 1e6  # 4 schedulers x 1 warp-instruction/clk
+        line["roofline"]["issue"] = {"achieved_warp_inst_per_s": ips, "peak": peak_ips, "frac": ips / peak_ips,
+                                     "source": "ncu smsp__inst_executed.sum per launch (profiles/) / live event time"}
     if not a.no_cpu_baseline and R.world == 1:
         cb = cpu_baseline(w, count, a.cpu_seconds)
         # parity of the bench's own configuration on the oracle's sample range

@@ -59,7 +59,13 @@ enum {
     XS_SEARCH_M2 = 6, /* unroll-only x2 of M (Fig. 7 "unroll" configuration)        */
     XS_SEARCH_M4 = 7, /* unroll-only x4                                             */
     XS_SEARCH_M8 = 8, /* unroll-only x8                                             */
-    XS_SEARCH_COUNT = 9
+    XS_SEARCH_W = 9,  /* warp-cooperative: in sorted modes a warp
+                         whose 32 lookups share a material finds L(q_min) and L(q_max) with
+                         two half-warp 17-ary searches over a per-nuclide separator tree
+                         (one 128 B node per level), then each lane runs Listing 1 inside
+                         [L(q_min), L(q_max)+1].  Nuclide grid only; elsewhere (unsorted,
+                         mixed-material warps, unionized/hash grids) it is U2.          */
+    XS_SEARCH_COUNT = 10
 };
 
 /* Lookup ordering (a pure reordering: results are invariant). */

@@ -130,6 +130,34 @@ __global__ void k_hash_table(int64_t bins, int32_t n_nuc, int32_t n, double du, 
     }
 }
 
+// separator tree: level d node `node` (path digits c_0..c_{d-1} in base 17) starts at
+// base = sum c_k * stride[k]; its key t is E[base + (t+1)*stride[d]] or +inf past the row
+__global__ void k_tree_build(int64_t n_nuc, int32_t n, int32_t levels, int4 stride_lo, int2 stride_hi,
+                             int4 off_lo, int2 off_hi, int64_t per_nuc, const double *__restrict__ E,
+                             double *__restrict__ keys)
+{
+    const int32_t stride[6] = {stride_lo.x, stride_lo.y, stride_lo.z, stride_lo.w, stride_hi.x, stride_hi.y};
+    const int32_t off[6] = {off_lo.x, off_lo.y, off_lo.z, off_lo.w, off_hi.x, off_hi.y};
+    const int64_t total = n_nuc * per_nuc;
+    for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < total; g += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t nuc = g / per_nuc;
+        const int32_t k = (int32_t)(g - nuc * per_nuc);
+        int d = 0;
+        while (d + 1 < levels && k >= off[d + 1])
+            d++;
+        const int32_t in_level = k - off[d];
+        const int32_t node = in_level / kTreeFan, t = in_level % kTreeFan;
+        int64_t base = 0;
+        int32_t rest = node;
+        for (int e = d - 1; e >= 0; e--) { // least significant digit = deepest level
+            base += (int64_t)(rest % 17) * stride[e];
+            rest /= 17;
+        }
+        const int64_t pos = base + (int64_t)(t + 1) * stride[d];
+        keys[g] = pos < n ? E[nuc * n + pos] : __longlong_as_double(0x7FF0000000000000ll);
+    }
+}
+
 // position-weighted checksum: h += word_k * (2*(offset+k)+1) over 32-bit words
 __global__ void k_checksum(const uint32_t *__restrict__ w, int64_t nwords, uint64_t offset, unsigned long long *out)
 {
@@ -220,6 +248,33 @@ void build_grid(Grid &g)
         cudaFree(tmp);
         tmp = nullptr;
 
+        // ---- separator tree over every nuclide row (XS_SEARCH_W)
+        {
+            int64_t R = n;
+            g.t_levels = 0;
+            int64_t nodes = 1, off = 0;
+            while (R > kTreeFan) {
+                const int64_t s = (R + 16) / 17; // ceil(R / 17)
+                g.t_stride[g.t_levels] = (int32_t)s;
+                g.t_off[g.t_levels] = (int32_t)off;
+                off += nodes * kTreeFan;
+                nodes *= 17;
+                g.t_levels++;
+                R = s;
+            }
+            g.t_leaf = (int32_t)R;
+            g.t_per_nuc = off;
+            if (off > 0) {
+                g.tkeys = dalloc<double>(g, g.n_nuc * off);
+                const int4 slo = make_int4(g.t_stride[0], g.t_stride[1], g.t_stride[2], g.t_stride[3]);
+                const int2 shi = make_int2(g.t_stride[4], g.t_stride[5]);
+                const int4 olo = make_int4(g.t_off[0], g.t_off[1], g.t_off[2], g.t_off[3]);
+                const int2 ohi = make_int2(g.t_off[4], g.t_off[5]);
+                k_tree_build<<<grid_blocks(g.n_nuc * off, tpb), tpb>>>(g.n_nuc, n, g.t_levels, slo, shi, olo, ohi,
+                                                                      off, g.E, g.tkeys);
+                XS_CUDA_TRY(cudaGetLastError());
+            }
+        }
         // ---- unionized grid (R4)
         if (g.grid_type == XS_UNIONIZED) {
             g.U = dalloc<double>(g, N);
@@ -257,6 +312,20 @@ void build_grid(Grid &g)
     XS_CUDA_TRY(cudaMemcpy(g.mats, mats.data(), mats.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
     XS_CUDA_TRY(cudaMemcpy(g.concs, concs.data(), concs.size() * sizeof(double), cudaMemcpyHostToDevice));
     XS_CUDA_TRY(cudaMemcpy(g.num_nucs_d, g.num_nucs, 12 * sizeof(int32_t), cudaMemcpyHostToDevice));
+    {
+        std::vector<NucRef> refs((size_t)12 * g.max_nucs, NucRef{nullptr, nullptr, nullptr, 0.0});
+        for (int m = 0; m < 12; m++)
+            for (int j = 0; j < g.num_nucs[m]; j++) {
+                const int64_t nuc = mats[(size_t)m * g.max_nucs + j];
+                NucRef &r = refs[(size_t)m * g.max_nucs + j];
+                r.E = g.E + nuc * g.n;
+                r.pts = g.pts + nuc * g.n * 6;
+                r.T = g.tkeys ? g.tkeys + nuc * g.t_per_nuc : nullptr;
+                r.conc = concs[(size_t)m * g.max_nucs + j];
+            }
+        g.refs = dalloc<NucRef>(g, (int64_t)refs.size());
+        XS_CUDA_TRY(cudaMemcpy(g.refs, refs.data(), refs.size() * sizeof(NucRef), cudaMemcpyHostToDevice));
+    }
 
     XS_CUDA_TRY(cudaMalloc(&g.stats_d, 8 * sizeof(uint64_t)));
     XS_CUDA_TRY(cudaMallocHost(&g.stats_h, 8 * sizeof(uint64_t)));
@@ -268,12 +337,14 @@ void free_grid(Grid &g)
 {
     cudaFree(g.E);
     cudaFree(g.pts);
+    cudaFree(g.tkeys);
     cudaFree(g.U);
     cudaFree(g.IDX);
     cudaFree(g.H);
     cudaFree(g.mats);
     cudaFree(g.concs);
     cudaFree(g.num_nucs_d);
+    cudaFree(g.refs);
     cudaFree(g.stats_d);
     if (g.stats_h)
         cudaFreeHost(g.stats_h);
@@ -330,12 +401,21 @@ GridView make_view(const Grid &g)
     v.mats = g.mats;
     v.concs = g.concs;
     v.num_nucs = g.num_nucs_d;
+    v.refs = (const NucRef *)g.refs;
     v.n = (int32_t)g.n;
     v.n_nuc = (int32_t)g.n_nuc;
     v.N = (int32_t)g.N;
     v.bins = (int32_t)g.bins;
     v.max_nucs = g.max_nucs;
     v.du = g.bins > 0 ? 1.0 / (double)g.bins : 0.0;
+    v.tkeys = g.tkeys;
+    v.t_levels = g.t_levels;
+    for (int d = 0; d < kTreeMaxLevels; d++) {
+        v.t_stride[d] = g.t_stride[d];
+        v.t_off[d] = g.t_off[d];
+    }
+    v.t_leaf = g.t_leaf;
+    v.t_per_nuc = (int32_t)g.t_per_nuc;
     return v;
 }
 

@@ -44,6 +44,46 @@ __device__ __forceinline__ int material_of(const uint32_t *mb, uint32_t j)
     return mat;
 }
 
+// ---- streaming loads: read once, keep them from evicting the grid out of L2 ----------------
+__device__ __forceinline__ uint64_t policy_evict_first()
+{
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+__device__ __forceinline__ uint32_t ld_stream(const uint32_t *a, uint64_t pol)
+{
+    uint32_t v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+    return v;
+}
+
+__device__ __forceinline__ double ld_stream(const double *a, uint64_t pol)
+{
+    double v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(a), "l"(pol));
+    return v;
+}
+
+// ---- nuclide j of material m --------------------------------------------------------------
+struct Row {
+    const double *E, *pts, *T;
+    double conc;
+};
+
+__device__ __forceinline__ Row load_row(const GridView &gv, int idx)
+{
+    const ulonglong2 *p = reinterpret_cast<const ulonglong2 *>(gv.refs + idx);
+    const ulonglong2 a = __ldg(p), b = __ldg(p + 1);
+    Row r;
+    r.E = opaque(reinterpret_cast<const double *>(a.x));
+    r.pts = opaque(reinterpret_cast<const double *>(a.y));
+    r.T = opaque(reinterpret_cast<const double *>(b.x));
+    r.conc = __longlong_as_double((long long)b.y);
+    return r;
+}
+
 // ---- the lower index of one (lookup, nuclide) pair ----------------------
 template <int GRID, int SEARCH>
 __device__ __forceinline__ int lower_index(const GridView &gv, const double *__restrict__ Ei, int nuc, double q,
@@ -78,15 +118,68 @@ __device__ __forceinline__ const double *nuclide_row(const GridView &gv, int nuc
     return opaque(gv.E + (size_t)nuc * (uint32_t)gv.n);
 }
 
+// ---- warp-cooperative bounds (XS_SEARCH_W) ----------------------------------
+// All 32 lanes of a warp whose lookups share a material call this for the same nuclide.
+// Lanes 0-15 find ub(q_lo) and lanes 16-31 ub(q_hi), ub(q) = #{k : E[k] <= q}: at each
+// level a half-warp loads one 16-key node (one 128 B line) of the separator tree, counts
+// the keys <= its query with one ballot, and descends into child c; the leaf compares
+// <= 16 consecutive energies.  Returns L(q_lo), L(q_hi) = clamp(ub - 1, 0, n-2) in every
+// lane, so each lane's L(q) lies in [L_lo, L_hi] (q_lo <= q <= q_hi, L monotone).
+__device__ __forceinline__ bool tree_usable(const GridView &gv) { return gv.tkeys != nullptr || gv.n <= kTreeFan; }
+
+__device__ __forceinline__ void warp_bounds(const GridView &gv, const double *__restrict__ Ei,
+                                            const double *__restrict__ T, double q_lo, double q_hi, int &L_lo,
+                                            int &L_hi)
+{
+    const int lane = threadIdx.x & 31, t = lane & 15;
+    const double qh = lane < 16 ? q_lo : q_hi;
+    const unsigned half = lane < 16 ? 0x0000FFFFu : 0xFFFF0000u;
+    int base = 0, node = 0;
+#pragma unroll
+    for (int d = 0; d < kTreeMaxLevels; d++) {
+        if (d < gv.t_levels) {
+            const double key = __ldg(T + (uint32_t)(gv.t_off[d] + node * kTreeFan + t));
+            const int c = __popc(__ballot_sync(0xffffffffu, key <= qh) & half);
+            base += c * gv.t_stride[d];
+            node = node * 17 + c;
+        }
+    }
+    const int pos = base + t;
+    const double key = (t < gv.t_leaf && pos < gv.n) ? __ldg(Ei + (uint32_t)pos)
+                                                     : __longlong_as_double(0x7FF0000000000000ll);
+    const int ub = base + __popc(__ballot_sync(0xffffffffu, key <= qh) & half);
+    const int ub_lo = __shfl_sync(0xffffffffu, ub, 0);
+    const int ub_hi = __shfl_sync(0xffffffffu, ub, 16);
+    L_lo = min(max(ub_lo - 1, 0), gv.n - 2);
+    L_hi = min(max(ub_hi - 1, 0), gv.n - 2);
+}
+
+__device__ __forceinline__ double warp_min(double v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+        v = fmin(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+
+__device__ __forceinline__ double warp_max(double v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+        v = fmax(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+
 // ---- interpolation + accumulation of one pair (reading R8) ------------------------------
 struct Acc {
     double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0, a4 = 0.0;
 };
 
 // 96 B gather: the 48 B records of points L and L+1, three 16 B loads each
-__device__ __forceinline__ void accumulate_pair(const GridView &gv, int nuc, int L, double q, double conc, Acc &A)
+__device__ __forceinline__ void accumulate_pair(const double *__restrict__ pts_row, int L, double q, double conc,
+                                                Acc &A)
 {
-    const double2 *p = reinterpret_cast<const double2 *>(gv.pts) + ((size_t)nuc * (uint32_t)gv.n + L) * 3;
+    const double2 *p = reinterpret_cast<const double2 *>(pts_row) + (uint32_t)L * 3;
     const double2 l0 = __ldg(p + 0), l1 = __ldg(p + 1), l2 = __ldg(p + 2);
     const double2 h0 = __ldg(p + 3), h1 = __ldg(p + 4), h2 = __ldg(p + 5);
     const double f = __ddiv_rn(__dsub_rn(h0.x, q), __dsub_rn(h0.x, l0.x));

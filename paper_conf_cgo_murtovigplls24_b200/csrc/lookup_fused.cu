@@ -1,7 +1,12 @@
 // lookup_fused.cu -- one thread per lookup, search + interpolation fused (XSBench's
 // event kernel shape).  Used for XS_SORT_NONE (sampling fused in: the
-// XSBench baseline order) and, with XS_FLAG_FUSED, for sorted lookups (the A/B against the
-// split path of lookup_split.cu).
+// XSBench baseline order) and, by default, for sorted lookups.
+//
+// The loop is warp-synchronous: each iteration a warp takes 32 consecutive lookup slots
+// (lanes past the end idle), so warp collectives are legal inside it.  With XS_SEARCH_W
+// on a nuclide grid, a warp whose 32 sorted lookups share one material searches each
+// nuclide cooperatively (warp_bounds) and every lane finishes with Listing 1 inside the
+// warp's window; any other warp runs the per-lane search.
 #include <algorithm>
 
 #include "lookup_common.cuh"
@@ -9,12 +14,20 @@
 namespace xs {
 
 constexpr int kFusedTpb = 256;
+#ifndef XS_W_MIN_BLOCKS
+#define XS_W_MIN_BLOCKS 4
+#endif
 
-template <int GRID, int SEARCH, bool SORTED>
-__global__ void __launch_bounds__(kFusedTpb, 4)
-    k_lookup(GridView gv, SampleView sv, SortedView so, Affine J_grid, double *__restrict__ out,
-             int32_t *__restrict__ out_idx, unsigned long long *__restrict__ stats)
+// OUTS: the call asked for macroscopic XS and/or indices; without it the bench/hash path
+// carries no output pointers (fewer live registers, no spills at 64 per thread)
+template <int GRID, int SEARCH, bool SORTED, bool OUTS>
+__global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BLOCKS : 4)
+    k_lookup(GridView gv, SampleView sv, SortedView so, Affine J_grid, double *__restrict__ out_,
+             int32_t *__restrict__ out_idx_, unsigned long long *__restrict__ stats)
 {
+    double *__restrict__ out = OUTS ? out_ : nullptr;
+    int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
+    constexpr bool kCoop = SORTED && SEARCH == XS_SEARCH_W && GRID == XS_NUCLIDE;
     __shared__ uint32_t s_mb[kMaterials + 1];
     if constexpr (SORTED) {
         if (threadIdx.x <= kMaterials)
@@ -24,75 +37,104 @@ __global__ void __launch_bounds__(kFusedTpb, 4)
     uint32_t my_hash = 0, my_pairs = 0;
     const int count = (int)sv.count;
     const int G = gridDim.x * blockDim.x;
-    int j = blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    const int j0 = blockIdx.x * blockDim.x + threadIdx.x;
     uint64_t s = 0;
     uint32_t r_next = 0;
     double q_next = 0.0;
+    const uint64_t pol = policy_evict_first();
     if constexpr (!SORTED) {
-        if (j < count)
-            s = lookup_state(sv, j);
-    } else if (j < count) {
-        r_next = __ldg(so.slot + j);
-        q_next = __ldg(so.q_of + r_next);
+        if (j0 < count)
+            s = lookup_state(sv, j0);
+    } else if (j0 < count) {
+        r_next = ld_stream(so.slot + j0, pol);
+        q_next = ld_stream(so.q_of + r_next, pol);
     }
-    for (; j < count; j += G) {
-        double q;
-        int mat;
-        uint32_t r;
-        if constexpr (SORTED) {
-            // the slot's lookup and energy were fetched one iteration ahead: the dependent
-            // random 8 B read of q_of overlaps this lookup's ~15-300 nuclide searches
-            q = q_next;
-            r = r_next;
-            if (j + G < count) {
-                r_next = __ldg(so.slot + j + G);
-                q_next = __ldg(so.q_of + r_next);
+    for (int jw = j0 - lane; jw < count; jw += G) { // warp-uniform trip count
+        const int j = jw + lane;
+        const bool active = j < count;
+        double q = 0.0;
+        int mat = 0;
+        uint32_t r = 0;
+        if (active) {
+            if constexpr (SORTED) {
+                // this slot's lookup and energy were fetched one iteration ahead: the
+                // dependent random 8 B read of q_of overlaps a whole lookup's searches
+                q = q_next;
+                r = r_next;
+                if (j + G < count) {
+                    r_next = ld_stream(so.slot + j + G, pol);
+                    q_next = ld_stream(so.q_of + r_next, pol);
+                }
+                mat = material_of(s_mb, (uint32_t)j);
+            } else {
+                sample_lookup(s, sv, q, mat);
+                r = (uint32_t)j;
+                s = lcg_apply(J_grid, s);
             }
-            mat = material_of(s_mb, (uint32_t)j);
-        } else {
-            sample_lookup(s, sv, q, mat);
-            r = (uint32_t)j;
-            s = lcg_apply(J_grid, s);
         }
-        const int nn = __ldg(gv.num_nucs + mat);
+        const int nn = active ? __ldg(gv.num_nucs + mat) : 0;
         const int row = mat * gv.max_nucs;
-        const int e_union = union_index<GRID, SEARCH>(gv, q);
         Acc A;
-        for (int jn = 0; jn < nn; jn++) {
-            const int nuc = __ldg(gv.mats + row + jn);
-            const double conc = __ldg(gv.concs + row + jn);
-            const int L = lower_index<GRID, SEARCH>(gv, nuclide_row(gv, nuc), nuc, q, e_union);
-            if (out_idx)
-                out_idx[(size_t)r * gv.max_nucs + jn] = L;
-            accumulate_pair(gv, nuc, L, q, conc, A);
+        bool coop = false;
+        if constexpr (kCoop) {
+            const int mat0 = __shfl_sync(0xffffffffu, mat, 0);
+            coop = __all_sync(0xffffffffu, active && mat == mat0) && tree_usable(gv);
         }
-        my_hash += verify(A);
-        my_pairs += (uint32_t)nn;
-        if (out)
-            store_macro(out, r, A);
+        if (coop) { // warp-uniform branch: all 32 lanes, same material, same nuclides
+            const double q_lo = warp_min(q), q_hi = warp_max(q);
+            for (int jn = 0; jn < nn; jn++) {
+                const Row rw = load_row(gv, row + jn);
+                int L_lo, L_hi;
+                warp_bounds(gv, rw.E, rw.T, q_lo, q_hi, L_lo, L_hi);
+                const int L = (L_lo == L_hi) ? L_lo : search<XS_SEARCH_U2>(rw.E, L_lo, L_hi + 1, q);
+                if (out_idx)
+                    out_idx[(size_t)r * gv.max_nucs + jn] = L;
+                accumulate_pair(rw.pts, L, q, rw.conc, A);
+            }
+        } else if (active) {
+            const int e_union = union_index<GRID, SEARCH>(gv, q);
+            for (int jn = 0; jn < nn; jn++) {
+                const Row rw = load_row(gv, row + jn);
+                const int nuc = (GRID == XS_NUCLIDE) ? 0 : __ldg(gv.mats + row + jn);
+                const int L = lower_index<GRID, SEARCH>(gv, rw.E, nuc, q, e_union);
+                if (out_idx)
+                    out_idx[(size_t)r * gv.max_nucs + jn] = L;
+                accumulate_pair(rw.pts, L, q, rw.conc, A);
+            }
+        }
+        if (active) {
+            my_hash += verify(A);
+            my_pairs += (uint32_t)nn;
+            if (out)
+                store_macro(out, r, A);
+        }
     }
     reduce_stats<kFusedTpb>(my_hash, my_pairs, stats);
 }
 
 using FusedFn = void (*)(GridView, SampleView, SortedView, Affine, double *, int32_t *, unsigned long long *);
 
-template <int GRID, int SEARCH> static FusedFn pick_s(bool sorted)
+template <int GRID, int SEARCH> static FusedFn pick_s(bool sorted, bool outs)
 {
-    return sorted ? k_lookup<GRID, SEARCH, true> : k_lookup<GRID, SEARCH, false>;
+    if (sorted)
+        return outs ? k_lookup<GRID, SEARCH, true, true> : k_lookup<GRID, SEARCH, true, false>;
+    return outs ? k_lookup<GRID, SEARCH, false, true> : k_lookup<GRID, SEARCH, false, false>;
 }
 
-template <int GRID> static FusedFn pick_g(int search, bool sorted)
+template <int GRID> static FusedFn pick_g(int search, bool sorted, bool outs)
 {
     switch (search) {
-    case XS_SEARCH_M: return pick_s<GRID, XS_SEARCH_M>(sorted);
-    case XS_SEARCH_U1: return pick_s<GRID, XS_SEARCH_U1>(sorted);
-    case XS_SEARCH_U2: return pick_s<GRID, XS_SEARCH_U2>(sorted);
-    case XS_SEARCH_U4: return pick_s<GRID, XS_SEARCH_U4>(sorted);
-    case XS_SEARCH_U8: return pick_s<GRID, XS_SEARCH_U8>(sorted);
-    case XS_SEARCH_B: return pick_s<GRID, XS_SEARCH_B>(sorted);
-    case XS_SEARCH_M2: return pick_s<GRID, XS_SEARCH_M2>(sorted);
-    case XS_SEARCH_M4: return pick_s<GRID, XS_SEARCH_M4>(sorted);
-    default: return pick_s<GRID, XS_SEARCH_M8>(sorted);
+    case XS_SEARCH_M: return pick_s<GRID, XS_SEARCH_M>(sorted, outs);
+    case XS_SEARCH_U1: return pick_s<GRID, XS_SEARCH_U1>(sorted, outs);
+    case XS_SEARCH_U2: return pick_s<GRID, XS_SEARCH_U2>(sorted, outs);
+    case XS_SEARCH_U4: return pick_s<GRID, XS_SEARCH_U4>(sorted, outs);
+    case XS_SEARCH_U8: return pick_s<GRID, XS_SEARCH_U8>(sorted, outs);
+    case XS_SEARCH_B: return pick_s<GRID, XS_SEARCH_B>(sorted, outs);
+    case XS_SEARCH_M2: return pick_s<GRID, XS_SEARCH_M2>(sorted, outs);
+    case XS_SEARCH_M4: return pick_s<GRID, XS_SEARCH_M4>(sorted, outs);
+    case XS_SEARCH_M8: return pick_s<GRID, XS_SEARCH_M8>(sorted, outs);
+    default: return pick_s<GRID, XS_SEARCH_W>(sorted, outs);
     }
 }
 
@@ -100,9 +142,10 @@ void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, c
                   const GridView &gv, const SampleView &sv, const SortedView &so, Affine J_grid, double *out,
                   int32_t *out_idx, unsigned long long *stats)
 {
-    FusedFn f = grid_type == XS_NUCLIDE     ? pick_g<XS_NUCLIDE>(search, sorted)
-                : grid_type == XS_UNIONIZED ? pick_g<XS_UNIONIZED>(search, sorted)
-                                            : pick_g<XS_HASH>(search, sorted);
+    const bool outs = out || out_idx;
+    FusedFn f = grid_type == XS_NUCLIDE     ? pick_g<XS_NUCLIDE>(search, sorted, outs)
+                : grid_type == XS_UNIONIZED ? pick_g<XS_UNIONIZED>(search, sorted, outs)
+                                            : pick_g<XS_HASH>(search, sorted, outs);
     f<<<blocks, tpb, 0, stream>>>(gv, sv, so, J_grid, out, out_idx, stats);
     XS_CUDA_TRY(cudaGetLastError());
 }

@@ -52,8 +52,9 @@ __global__ void __launch_bounds__(kSearchTpb, 8)
         const int row = mat * gv.max_nucs;
         const int e_union = union_index<GRID, SEARCH>(gv, q);
         for (int jn = 0; jn < nn; jn++) {
-            const int nuc = __ldg(gv.mats + row + jn);
-            dst[(size_t)jn * stride] = lower_index<GRID, SEARCH>(gv, nuclide_row(gv, nuc), nuc, q, e_union);
+            const Row rw = load_row(gv, row + jn);
+            const int nuc = (GRID == XS_NUCLIDE) ? 0 : __ldg(gv.mats + row + jn);
+            dst[(size_t)jn * stride] = lower_index<GRID, SEARCH>(gv, rw.E, nuc, q, e_union);
         }
     }
 }
@@ -77,12 +78,11 @@ __global__ void __launch_bounds__(kInterpTpb, 2)
         const uint32_t r = (out || out_idx) ? so.slot[j] : 0u;
         Acc A;
         for (int jn = 0; jn < nn; jn++) {
-            const int nuc = __ldg(gv.mats + row + jn);
-            const double conc = __ldg(gv.concs + row + jn);
+            const Row rw = load_row(gv, row + jn);
             const int L = __ldg(src + (size_t)jn * stride);
             if (out_idx)
                 out_idx[(size_t)r * gv.max_nucs + jn] = L;
-            accumulate_pair(gv, nuc, L, q, conc, A);
+            accumulate_pair(rw.pts, L, q, rw.conc, A);
         }
         my_hash += verify(A);
         my_pairs += (uint32_t)nn;
@@ -105,7 +105,8 @@ template <int GRID> static SearchKFn pick_g(int search)
     case XS_SEARCH_B: return k_search<GRID, XS_SEARCH_B>;
     case XS_SEARCH_M2: return k_search<GRID, XS_SEARCH_M2>;
     case XS_SEARCH_M4: return k_search<GRID, XS_SEARCH_M4>;
-    default: return k_search<GRID, XS_SEARCH_M8>;
+    case XS_SEARCH_M8: return k_search<GRID, XS_SEARCH_M8>;
+    default: return k_search<GRID, XS_SEARCH_W>;
     }
 }
 

@@ -49,7 +49,8 @@ template <int GRID> static SearchPtsFn pick_pts(int search)
     case XS_SEARCH_B: return k_search_points<GRID, XS_SEARCH_B>;
     case XS_SEARCH_M2: return k_search_points<GRID, XS_SEARCH_M2>;
     case XS_SEARCH_M4: return k_search_points<GRID, XS_SEARCH_M4>;
-    default: return k_search_points<GRID, XS_SEARCH_M8>;
+    case XS_SEARCH_M8: return k_search_points<GRID, XS_SEARCH_M8>;
+    default: return k_search_points<GRID, XS_SEARCH_W>;
     }
 }
 

@@ -33,6 +33,8 @@ void clear_error();
 
 constexpr int kMaterials = 12;
 constexpr int kMaxEnergyBins = 4096;
+constexpr int kTreeFan = 16;     // separator keys per node: one 128 B line
+constexpr int kTreeMaxLevels = 6; // n < 17^6 * 16 for every n_gridpoints < 2^31
 
 // ---- the grid in HBM -----------------------------------------------------
 //   E   [n_nuc][n]      fp64  search keys, SoA (8 B stride: the probes of Listing 1)
@@ -54,12 +56,21 @@ struct Grid {
 
     double *E = nullptr;
     double *pts = nullptr;
+    // separator tree of every nuclide row (XS_SEARCH_W): level d has
+    // 17^d nodes of 16 keys; node keys are E at base + (t+1)*stride[d] (+inf past n)
+    double *tkeys = nullptr;
+    int32_t t_levels = 0;
+    int32_t t_stride[kTreeMaxLevels] = {};
+    int32_t t_off[kTreeMaxLevels] = {};
+    int32_t t_leaf = 0;       // elements probed at the leaf (<= 16)
+    int64_t t_per_nuc = 0;    // keys per nuclide
     double *U = nullptr;
     int32_t *IDX = nullptr;
     int32_t *H = nullptr;
     int32_t *mats = nullptr;
     double *concs = nullptr;
     int32_t *num_nucs_d = nullptr;
+    void *refs = nullptr;            // NucRef [12][max_nucs]: row pointers + conc per (mat, j)
 
     // per-grid scratch (grown on demand; calls on one grid are serialised by the caller)
     uint64_t *stats_d = nullptr;     // [4] hash, pairs
@@ -95,6 +106,15 @@ struct DeviceGuard {
 };
 
 // ---- kernel arguments ----------------------------------------------------------------
+// Everything the lookup loop needs about nuclide j of material m, precomputed at grid
+// creation so the loop does one 32 B broadcast load instead of 64-bit row arithmetic.
+struct NucRef {
+    const double *E;   // energy row of the nuclide            (E + nuc * n)
+    const double *pts; // 48 B point records of the nuclide    (pts + nuc * n * 6)
+    const double *T;   // separator tree of the nuclide, or NULL
+    double conc;       // concs[m][j]
+};
+
 struct GridView {
     const double *__restrict__ E;
     const double *__restrict__ pts;
@@ -104,13 +124,19 @@ struct GridView {
     const int32_t *__restrict__ mats;
     const double *__restrict__ concs;
     const int32_t *__restrict__ num_nucs;
+    const NucRef *__restrict__ refs;
     int32_t n;        // gridpoints per nuclide
     int32_t n_nuc;
     int32_t N;        // n_nuc * n
     int32_t bins;
     int32_t max_nucs;
-    int32_t pad_;
+    int32_t t_levels;
     double du;        // 1.0 / bins
+    const double *__restrict__ tkeys;
+    int32_t t_stride[kTreeMaxLevels];
+    int32_t t_off[kTreeMaxLevels];
+    int32_t t_leaf;
+    int32_t t_per_nuc;
 };
 
 struct SampleView {

@@ -7,10 +7,10 @@ import paper_conf_cgo_murtovigplls24_b200 as xs
 from xs_workloads import WORKLOADS, GRID_SEED, LOOKUP_SEED
 w = WORKLOADS[sys.argv[1]]
 search, sort = sys.argv[2], sys.argv[3]
-fused = os.environ.get("XS_FUSED", "0") == "1"
+split = os.environ.get("XS_SPLIT", "0") == "1"
 reps = int(sys.argv[4]) if len(sys.argv) > 4 else 3
 n = int(sys.argv[5]) if len(sys.argv) > 5 else w.lookups
 g = xs.Grid(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED)
 for _ in range(reps):
-    st = g.lookup_range(0, n, LOOKUP_SEED, search=search, sort=sort, split=not fused)
+    st = g.lookup_range(0, n, LOOKUP_SEED, search=search, sort=sort, split=split)
 print("hash", st.hash, "device_ms", st.device_ms)
