@@ -119,7 +119,7 @@ typedef struct xs_grid_info {
     int32_t num_nucs[12];
 } xs_grid_info;
 
-/* Fill *opts with the defaults (best unmerged variant, XS_SORT_MATERIAL_ENERGY). */
+/* Fill *opts with the defaults: XS_SEARCH_W, XS_SORT_MATERIAL_ENERGY, legacy stream, no flags. */
 void xs_opts_default(xs_opts *opts);
 
 /* Build a grid on the current CUDA device:

@@ -361,6 +361,14 @@ void free_grid(Grid &g)
     for (auto &e : g.ev)
         if (e)
             cudaEventDestroy(e);
+    for (int b = 0; b < 2; b++) {
+        if (g.ev_done[b])
+            cudaEventDestroy(g.ev_done[b]);
+        if (g.ev_copied[b])
+            cudaEventDestroy(g.ev_copied[b]);
+    }
+    if (g.copy_stream)
+        cudaStreamDestroy(g.copy_stream);
 }
 
 uint64_t grid_checksum(const Grid &g)

@@ -100,7 +100,7 @@ template <class T> static void grow(T *&p, int64_t &cap, int64_t need)
 
 constexpr int64_t kChunkFused = int64_t(1) << 28;  // uint32 slots
 constexpr int64_t kChunkSplit = int64_t(1) << 25;  // pair buffer <= 33.5M x 321 x 4 B
-constexpr int64_t kChunkHost = int64_t(1) << 23;   // staging for host outputs
+constexpr int64_t kChunkHost = int64_t(1) << 22;   // staging for host outputs (x2 buffers)
 
 void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
                  int32_t *out_idx, xs_stats *st)
@@ -124,8 +124,18 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
     int launches = 0;
     double sample_ms = 0, lookup_ms = 0, search_ms = 0, copy_ms = 0;
 
-    if (host_out)
-        grow(g.stage, g.stage_cap, std::min(count, chunk) * 5);
+    if (host_out) {
+        grow(g.stage, g.stage_cap, std::min(count, chunk) * 5 * 2);
+        if (!g.copy_stream) {
+            XS_CUDA_TRY(cudaStreamCreateWithFlags(&g.copy_stream, cudaStreamNonBlocking));
+            for (int b = 0; b < 2; b++) {
+                XS_CUDA_TRY(cudaEventCreateWithFlags(&g.ev_done[b], cudaEventDisableTiming));
+                XS_CUDA_TRY(cudaEventCreateWithFlags(&g.ev_copied[b], cudaEventDisableTiming));
+            }
+        }
+    }
+    bool copied_pending[2] = {false, false};
+    const int64_t stage_half = std::min(count, chunk) * 5;
     if (!g.mb_h)
         XS_CUDA_TRY(cudaMallocHost(&g.mb_h, 32 * sizeof(uint32_t)));
 
@@ -135,10 +145,14 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         XS_CUDA_TRY(cudaMemsetAsync(out_idx, 0xFF, (size_t)count * g.max_nucs * sizeof(int32_t), stream));
     unsigned long long *stats = (unsigned long long *)g.stats_d;
 
-    for (int64_t c0 = 0; c0 < count; c0 += chunk) {
+    for (int64_t c0 = 0, ci = 0; c0 < count; c0 += chunk, ci++) {
         const int64_t cn = std::min(chunk, count - c0);
         const SampleView sv = make_sample_view(g, seed, first + c0, cn);
-        double *outp = out_macro ? (host_out ? g.stage : out_macro + c0 * 5) : nullptr;
+        const int buf = (int)(ci & 1);
+        double *stage = g.stage + buf * stage_half;
+        if (host_out && copied_pending[buf]) // the copy out of this buffer must be done
+            XS_CUDA_TRY(cudaStreamWaitEvent(stream, g.ev_copied[buf], 0));
+        double *outp = out_macro ? (host_out ? stage : out_macro + c0 * 5) : nullptr;
         int32_t *idxp = out_idx ? out_idx + c0 * g.max_nucs : nullptr;
         SortedView so{};
         XS_CUDA_TRY(cudaEventRecord(g.ev[1], stream));
@@ -179,9 +193,14 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             launches += 2;
         }
         XS_CUDA_TRY(cudaEventRecord(g.ev[4], stream));
-        if (host_out)
-            XS_CUDA_TRY(cudaMemcpyAsync(out_macro + c0 * 5, g.stage, (size_t)cn * 5 * sizeof(double),
-                                        cudaMemcpyDeviceToHost, stream));
+        if (host_out) { // D2H on the copy stream, overlapped with the next chunk's kernels
+            XS_CUDA_TRY(cudaEventRecord(g.ev_done[buf], stream));
+            XS_CUDA_TRY(cudaStreamWaitEvent(g.copy_stream, g.ev_done[buf], 0));
+            XS_CUDA_TRY(cudaMemcpyAsync(out_macro + c0 * 5, stage, (size_t)cn * 5 * sizeof(double),
+                                        cudaMemcpyDeviceToHost, g.copy_stream));
+            XS_CUDA_TRY(cudaEventRecord(g.ev_copied[buf], g.copy_stream));
+            copied_pending[buf] = true;
+        }
         XS_CUDA_TRY(cudaEventRecord(g.ev[5], stream));
         if (timing) {
             XS_CUDA_TRY(cudaStreamSynchronize(stream));
@@ -189,6 +208,11 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             cudaEventElapsedTime(&a, g.ev[1], g.ev[2]);
             cudaEventElapsedTime(&b, g.ev[2], g.ev[4]);
             cudaEventElapsedTime(&c, g.ev[2], g.ev[3]);
+            if (host_out) { // timing mode serialises: time the chunk's copy on its own
+                XS_CUDA_TRY(cudaStreamSynchronize(g.copy_stream));
+                cudaEventRecord(g.ev[5], stream);
+                XS_CUDA_TRY(cudaStreamSynchronize(stream));
+            }
             cudaEventElapsedTime(&d, g.ev[4], g.ev[5]);
             sample_ms += a;
             lookup_ms += b;
@@ -196,6 +220,9 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             copy_ms += d;
         }
     }
+    for (int b = 0; b < 2; b++) // the call's stream covers every outstanding copy
+        if (copied_pending[b])
+            XS_CUDA_TRY(cudaStreamWaitEvent(stream, g.ev_copied[b], 0));
     XS_CUDA_TRY(cudaMemcpyAsync(g.stats_h, g.stats_d, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, stream));
     XS_CUDA_TRY(cudaEventRecord(g.ev[6], stream));
     XS_CUDA_TRY(cudaStreamSynchronize(stream));

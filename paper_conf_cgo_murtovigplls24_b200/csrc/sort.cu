@@ -52,14 +52,50 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, int nb
         h[k] = sh[k];
 }
 
+// per bucket k: exclusive scan over the CTAs, in place; total[k] = the bucket's size.
+// 4 threads per bucket (adjacent lanes) each own a quarter of the CTA rows, so the
+// dependent chain of row loads is 4x shorter; loads are batched by 8.
+constexpr int kColSplit = 4;
+
+__device__ __forceinline__ uint32_t colsum(const uint32_t *hist, int K, int k, int c0, int c1)
+{
+    uint32_t run = 0;
+    int c = c0;
+    for (; c + 8 <= c1; c += 8) {
+        uint32_t v[8];
+#pragma unroll
+        for (int u = 0; u < 8; u++)
+            v[u] = hist[(int64_t)(c + u) * K + k];
+#pragma unroll
+        for (int u = 0; u < 8; u++)
+            run += v[u];
+    }
+    for (; c < c1; c++)
+        run += hist[(int64_t)c * K + k];
+    return run;
+}
+
 __global__ void k_bucket_colscan(int K, int ctas, uint32_t *hist, uint32_t *__restrict__ total)
 {
-    const int k = blockIdx.x * blockDim.x + threadIdx.x;
-    if (k >= K)
+    const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+    const int k = tid / kColSplit, part = tid % kColSplit;
+    const int per = (ctas + kColSplit - 1) / kColSplit;
+    const int c0 = min(part * per, ctas), c1 = min(c0 + per, ctas);
+    const bool valid = k < K;
+    const uint32_t mine = valid ? colsum(hist, K, k, c0, c1) : 0u;
+    // exclusive scan of the 4 partial sums (lanes 4k'..4k'+3 of the warp)
+    uint32_t incl = mine;
+#pragma unroll
+    for (int o = 1; o < kColSplit; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o, kColSplit);
+        if (part >= o)
+            incl += t;
+    }
+    if (!valid)
         return;
-    uint32_t run = 0;
-    int c = 0;
-    for (; c + 8 <= ctas; c += 8) {
+    uint32_t run = incl - mine;
+    int c = c0;
+    for (; c + 8 <= c1; c += 8) {
         uint32_t v[8];
 #pragma unroll
         for (int u = 0; u < 8; u++)
@@ -70,58 +106,66 @@ __global__ void k_bucket_colscan(int K, int ctas, uint32_t *hist, uint32_t *__re
             run += v[u];
         }
     }
-    for (; c < ctas; c++) {
+    for (; c < c1; c++) {
         const uint32_t v = hist[(int64_t)c * K + k];
         hist[(int64_t)c * K + k] = run;
         run += v;
     }
-    total[k] = run;
+    if (part == kColSplit - 1)
+        total[k] = run;
 }
 
+// one CTA: exclusive scan of base[0..K) in place.  All K values are staged in shared
+// memory with coalesced loads, each thread scans a contiguous run of ceil(K/1024), a
+// block scan combines the runs, and the results go back coalesced.  Then
+// base[K + m] = first slot of material m (m = 0..11), base[K + 12] = count.
 __global__ void __launch_bounds__(1024) k_bucket_base(int K, int nb_log2, uint32_t *__restrict__ base)
 {
+    extern __shared__ uint32_t sv[];
     __shared__ uint32_t wsum[32];
-    __shared__ uint32_t carry;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    if (threadIdx.x == 0)
-        carry = 0;
+    for (int k = threadIdx.x; k < K; k += 1024)
+        sv[k] = base[k];
     __syncthreads();
-    for (int r0 = 0; r0 < K; r0 += 1024) {
-        const int k = r0 + threadIdx.x;
-        const uint32_t v = k < K ? base[k] : 0u;
-        uint32_t incl = v;
+    const int per = (K + 1023) / 1024;
+    const int b0 = min((int)threadIdx.x * per, K), b1 = min(b0 + per, K);
+    uint32_t mine = 0;
+    for (int k = b0; k < b1; k++)
+        mine += sv[k];
+    uint32_t incl = mine;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o)
+            incl += t;
+    }
+    if (lane == 31)
+        wsum[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        uint32_t w = wsum[lane];
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+            const uint32_t t = __shfl_up_sync(0xffffffffu, w, o);
             if (lane >= o)
-                incl += t;
+                w += t;
         }
-        if (lane == 31)
-            wsum[wid] = incl;
-        __syncthreads();
-        if (wid == 0) {
-            uint32_t w = wsum[lane];
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t t = __shfl_up_sync(0xffffffffu, w, o);
-                if (lane >= o)
-                    w += t;
-            }
-            wsum[lane] = w;
-        }
-        __syncthreads();
-        const uint32_t c0 = carry;
-        if (k < K)
-            base[k] = c0 + incl - v + (wid ? wsum[wid - 1] : 0u);
-        __syncthreads();
-        if (threadIdx.x == 0)
-            carry = c0 + wsum[31];
-        __syncthreads();
+        wsum[lane] = w;
     }
+    __syncthreads();
+    uint32_t run = incl - mine + (wid ? wsum[wid - 1] : 0u);
+    for (int k = b0; k < b1; k++) {
+        const uint32_t v = sv[k];
+        sv[k] = run;
+        run += v;
+    }
+    __syncthreads();
+    for (int k = threadIdx.x; k < K; k += 1024)
+        base[k] = sv[k];
     if (threadIdx.x < kMaterials)
-        base[K + threadIdx.x] = base[threadIdx.x << nb_log2];
+        base[K + threadIdx.x] = sv[threadIdx.x << nb_log2];
     if (threadIdx.x == 0)
-        base[K + kMaterials] = carry;
+        base[K + kMaterials] = wsum[31];
 }
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int nb_log2, int per_cta, int count,
@@ -138,10 +182,10 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int nb_log2, int pe
     __syncthreads();
     const int beg = blockIdx.x * per_cta;
     const int end = min(beg + per_cta, count);
-    for (int j = beg + threadIdx.x; j < end; j += kSortTpb) {
-        const uint32_t pos = atomicAdd(&sh[key_of[j]], 1u);
-        slot_of[pos] = (uint32_t)j;
-    }
+    // (recording each lookup's rank in the count pass to drop these atomics was measured
+    // slower: the scatter is bound by its random 4 B stores, not by the atomics)
+    for (int j = beg + threadIdx.x; j < end; j += kSortTpb)
+        slot_of[atomicAdd(&sh[key_of[j]], 1u)] = (uint32_t)j;
 }
 
 __global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of, const double *__restrict__ q_of,
@@ -196,6 +240,7 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gat
         const int bytes = kMaterials * kMaxEnergyBins * 4;
         XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_count, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
         XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+        XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_base, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
         smem_set[g.device & 63] = true;
     }
     const int64_t cn = sv.count;
@@ -207,8 +252,8 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gat
     const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
     const size_t smem = (size_t)K * 4;
     k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, nb_log2, per_cta, J, g.hist, g.sq, g.skey);
-    k_bucket_colscan<<<(K + 127) / 128, 128, 0, stream>>>(K, ctas, g.hist, g.base);
-    k_bucket_base<<<1, 1024, 0, stream>>>(K, nb_log2, g.base);
+    k_bucket_colscan<<<(K * kColSplit + 127) / 128, 128, 0, stream>>>(K, ctas, g.hist, g.base);
+    k_bucket_base<<<1, 1024, smem, stream>>>(K, nb_log2, g.base);
     k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(nb_log2, per_cta, (int)cn, g.hist, g.base, g.skey, g.si);
     XS_CUDA_TRY(cudaGetLastError());
     if (!with_gather)

@@ -85,8 +85,10 @@ struct Grid {
     uint32_t *hist = nullptr;        // per-CTA bucket histograms [ctas][K]
     uint32_t *base = nullptr;        // [K + 16]: bucket bases, then material bases
     int64_t cap = 0, hist_cap = 0;
-    double *stage = nullptr;         // device staging for host outputs
+    double *stage = nullptr;         // device staging for host outputs: 2 buffers
     int64_t stage_cap = 0;
+    cudaStream_t copy_stream = nullptr; // D2H of staged outputs, overlapped with compute
+    cudaEvent_t ev_done[2] = {}, ev_copied[2] = {};
     cudaEvent_t ev[8] = {};
 };
 

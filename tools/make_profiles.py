@@ -31,7 +31,7 @@ def main():
             rd = to_mb(num("dram__bytes_read.sum") or 0, u.get("dram__bytes_read.sum", "")) * 1e6
             wr = to_mb(num("dram__bytes_write.sum") or 0, u.get("dram__bytes_write.sum", "")) * 1e6
             dur = num("gpu__time_duration.sum")
-            dur_us = dur * {"nsecond": 1e-3, "usecond": 1, "msecond": 1e3}.get(u.get("gpu__time_duration.sum", ""), 1e-3)
+            dur_us = dur * {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1, "us": 1, "msecond": 1e3, "ms": 1e3}.get(u.get("gpu__time_duration.sum", ""), 1e-3)
             inst = num("smsp__inst_executed.sum")
             stalls = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): num(k) or 0 for k in hdr
                       if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("not_issued")}
@@ -46,7 +46,7 @@ def main():
                    f"| achieved occupancy % | {num('sm__warps_active.avg.pct_of_peak_sustained_active')} |",
                    f"| registers / thread | {num('launch__registers_per_thread')} |",
                    f"| L1 hit % / L2 hit % | {num('l1tex__t_sector_hit_rate.pct')} / {num('lts__t_sector_hit_rate.pct')} |",
-                   f"| DRAM throughput % of peak | {num('dram__throughput.avg.pct_of_peak_sustained_elapsed')} |",
+                   f"| DRAM throughput % of peak | {num('gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed')} |",
                    f"| threads per warp instruction | {num('smsp__thread_inst_executed_per_inst_executed.ratio')} |",
                    f"| branch targets uniform % | {num('smsp__sass_average_branch_targets_threads_uniform.pct')} |",
                    f"| FP64 pipe % | {num('sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active')} |",

@@ -6,7 +6,7 @@ KEYS = [
     ("gpu__time_duration.sum", "dur_us", 1e-3),
     ("dram__bytes_read.sum", "dram_rd_MB", None),
     ("dram__bytes_write.sum", "dram_wr_MB", None),
-    ("dram__throughput.avg.pct_of_peak_sustained_elapsed", "dram_pct", 1),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "dram_pct", 1),
     ("lts__t_sector_hit_rate.pct", "l2_hit_pct", 1),
     ("l1tex__t_sector_hit_rate.pct", "l1_hit_pct", 1),
     ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm_pct", 1),
@@ -49,7 +49,7 @@ def main():
                 if sc is None:
                     v = to_mb(v, u.get(k, ""))
                 elif k == "gpu__time_duration.sum":
-                    v = v * ({"nsecond": 1e-3, "usecond": 1, "msecond": 1e3}.get(u.get(k, ""), 1e-3))
+                    v = v * ({"nsecond": 1e-3, "ns": 1e-3, "usecond": 1, "us": 1, "msecond": 1e3, "ms": 1e3}.get(u.get(k, ""), 1e-3))
                 item[short] = round(v, 3)
         if "--stalls" in sys.argv:
             st = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): float(d[k].replace(",", "") or 0)
