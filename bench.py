@@ -47,13 +47,13 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="small", choices=sorted(WORKLOADS))
     p.add_argument("--lookups", type=int, default=0, help="override lookups per GPU")
-    p.add_argument("--search", default="W")
+    p.add_argument("--search", default="H")
     p.add_argument("--sort", default="material_energy")
     p.add_argument("--energy-bins", type=int, default=0)
     p.add_argument("--no-flush", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--ab", default="M,U1,U2,U4,U8,B,W", help="search variants for the A/B sub-object ('' = off)")
+    p.add_argument("--ab", default="M,U1,U2,U4,U8,B,W,H", help="search variants for the A/B sub-object ('' = off)")
     p.add_argument("--ab-steps", type=int, default=5)
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target wall time of the CPU sample")
     return p.parse_args()

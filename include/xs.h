@@ -65,7 +65,13 @@ enum {
                          (one 128 B node per level), then each lane runs Listing 1 inside
                          [L(q_min), L(q_max)+1].  Nuclide grid only; elsewhere (unsorted,
                          mixed-material warps, unionized/hash grids) it is U2.          */
-    XS_SEARCH_COUNT = 10
+    XS_SEARCH_H = 10, /* bin-bounded: per nuclide a table Tb[b] = L(b / 2^k), b = 0..2^k,
+                         2^k >= n_gridpoints (built at grid creation); q*2^k is exact, so
+                         L(q) lies in [Tb[b], Tb[b+1]] for b = floor(q*2^k) and Listing 1
+                         (U2) runs on that window -- usually 1-2 points.  XSBench's hash-
+                         grid idea (R7) at power-of-two resolution.  Nuclide grid only;
+                         elsewhere it is U2.                                              */
+    XS_SEARCH_COUNT = 11
 };
 
 /* Lookup ordering (a pure reordering: results are invariant). */
@@ -87,8 +93,10 @@ typedef struct xs_opts {
     int32_t sort;        /* XS_SORT_*                                                   */
     void *stream;        /* cudaStream_t, NULL = legacy default stream                  */
     int32_t block;       /* threads per CTA of the lookup kernel: 0 = default (256)     */
-    int32_t energy_bins; /* energy buckets per material for XS_SORT_MATERIAL_ENERGY:
-                            power of two in [1, 4096]; 0 = default (4096)               */
+    int32_t energy_bins; /* XS_SORT_MATERIAL_ENERGY: energy buckets per material on average,
+                            power of two in [1, 4096]; 0 = default (4096).  The 12 x
+                            energy_bins buckets are shared out in proportion to each
+                            material's expected (lookup, nuclide) pairs                 */
     uint32_t flags;      /* XS_FLAG_*                                                   */
     int32_t reserved;
 } xs_opts;
@@ -119,7 +127,7 @@ typedef struct xs_grid_info {
     int32_t num_nucs[12];
 } xs_grid_info;
 
-/* Fill *opts with the defaults: XS_SEARCH_W, XS_SORT_MATERIAL_ENERGY, legacy stream, no flags. */
+/* Fill *opts with the defaults: XS_SEARCH_H, XS_SORT_MATERIAL_ENERGY, legacy stream, no flags. */
 void xs_opts_default(xs_opts *opts);
 
 /* Build a grid on the current CUDA device:

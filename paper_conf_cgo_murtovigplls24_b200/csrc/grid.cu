@@ -158,6 +158,20 @@ __global__ void k_tree_build(int64_t n_nuc, int32_t n, int32_t levels, int4 stri
     }
 }
 
+// bin bounds: B[nuc][b] = L_nuc(b / 2^b_log2), b = 0 .. 2^b_log2 (the energy is exact)
+__global__ void k_bounds_build(int64_t n_nuc, int32_t n, int32_t b_log2, const double *__restrict__ E,
+                               int32_t *__restrict__ B)
+{
+    const int64_t per = ((int64_t)1 << b_log2) + 1;
+    const int64_t total = n_nuc * per;
+    const double scale = 1.0 / (double)((int64_t)1 << b_log2);
+    for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < total; g += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t nuc = g / per;
+        const int64_t b = g - nuc * per;
+        B[g] = search_M<1>(E + nuc * n, 0, n - 1, __dmul_rn((double)b, scale));
+    }
+}
+
 // position-weighted checksum: h += word_k * (2*(offset+k)+1) over 32-bit words
 __global__ void k_checksum(const uint32_t *__restrict__ w, int64_t nwords, uint64_t offset, unsigned long long *out)
 {
@@ -275,6 +289,19 @@ void build_grid(Grid &g)
                 XS_CUDA_TRY(cudaGetLastError());
             }
         }
+        // ---- bin bounds over every nuclide row (XS_SEARCH_H): 2^k >= n bins, capped
+        {
+            int b_log2 = 1;
+            while ((int64_t(1) << b_log2) < g.n && b_log2 < 20)
+                b_log2++;
+            const int64_t per = (int64_t(1) << b_log2) + 1;
+            if (g.n_nuc * per < (int64_t(1) << 31)) {
+                g.b_log2 = b_log2;
+                g.bnd = dalloc<int32_t>(g, g.n_nuc * per);
+                k_bounds_build<<<grid_blocks(g.n_nuc * per, tpb), tpb>>>(g.n_nuc, n, b_log2, g.E, g.bnd);
+                XS_CUDA_TRY(cudaGetLastError());
+            }
+        }
         // ---- unionized grid (R4)
         if (g.grid_type == XS_UNIONIZED) {
             g.U = dalloc<double>(g, N);
@@ -313,7 +340,7 @@ void build_grid(Grid &g)
     XS_CUDA_TRY(cudaMemcpy(g.concs, concs.data(), concs.size() * sizeof(double), cudaMemcpyHostToDevice));
     XS_CUDA_TRY(cudaMemcpy(g.num_nucs_d, g.num_nucs, 12 * sizeof(int32_t), cudaMemcpyHostToDevice));
     {
-        std::vector<NucRef> refs((size_t)12 * g.max_nucs, NucRef{nullptr, nullptr, nullptr, 0.0});
+        std::vector<NucRef> refs((size_t)12 * g.max_nucs, NucRef{nullptr, nullptr, nullptr, nullptr, 0.0, 0});
         for (int m = 0; m < 12; m++)
             for (int j = 0; j < g.num_nucs[m]; j++) {
                 const int64_t nuc = mats[(size_t)m * g.max_nucs + j];
@@ -321,7 +348,9 @@ void build_grid(Grid &g)
                 r.E = g.E + nuc * g.n;
                 r.pts = g.pts + nuc * g.n * 6;
                 r.T = g.tkeys ? g.tkeys + nuc * g.t_per_nuc : nullptr;
+                r.B = g.bnd ? g.bnd + nuc * ((int64_t(1) << g.b_log2) + 1) : nullptr;
                 r.conc = concs[(size_t)m * g.max_nucs + j];
+                r.nuc = nuc;
             }
         g.refs = dalloc<NucRef>(g, (int64_t)refs.size());
         XS_CUDA_TRY(cudaMemcpy(g.refs, refs.data(), refs.size() * sizeof(NucRef), cudaMemcpyHostToDevice));
@@ -338,6 +367,7 @@ void free_grid(Grid &g)
     cudaFree(g.E);
     cudaFree(g.pts);
     cudaFree(g.tkeys);
+    cudaFree(g.bnd);
     cudaFree(g.U);
     cudaFree(g.IDX);
     cudaFree(g.H);
@@ -424,6 +454,8 @@ GridView make_view(const Grid &g)
     }
     v.t_leaf = g.t_leaf;
     v.t_per_nuc = (int32_t)g.t_per_nuc;
+    v.b_log2 = g.bnd ? g.b_log2 : 0;
+    v.bnd = g.bnd;
     return v;
 }
 

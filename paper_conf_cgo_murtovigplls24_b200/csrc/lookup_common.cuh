@@ -27,11 +27,22 @@ __device__ __forceinline__ uint64_t lookup_state(const SampleView &sv, int64_t j
     return lcg_apply(lcg_jump(2 * (uint64_t)(sv.first + j)), sv.seed);
 }
 
-__device__ __forceinline__ int energy_bucket(double q, int nb_log2)
+// Sort buckets: material m owns keys [kbase[m], kbase[m] + nb[m]), nb[m] proportional to
+// its expected share of (lookup, nuclide) pairs, so the material that dominates the cost
+// gets the finest energy resolution.  Any key assignment is a valid ordering.
+struct BucketPlan {
+    int K;
+    int nb[kMaterials];
+    int kbase[kMaterials + 1];
+};
+
+// nb / kbase are read from shared memory: indexed by a per-lane material, a parameter-bank
+// read would serialise over the distinct materials of the warp
+__device__ __forceinline__ int bucket_key(const int *s_nb, const int *s_kbase, int mat, double q)
 {
-    const int nb = 1 << nb_log2;
-    const int b = (int)__dmul_rn(q, (double)nb); // exact: nb is a power of two
-    return b < nb - 1 ? b : nb - 1;              // q may be exactly 1.0 (R7)
+    const int nb = s_nb[mat];
+    const int b = (int)__dmul_rn(q, (double)nb);
+    return s_kbase[mat] + (b < nb - 1 ? b : nb - 1); // q may be exactly 1.0 (R7)
 }
 
 // material of sorted position j: the number of later materials whose first slot is <= j
@@ -69,27 +80,58 @@ __device__ __forceinline__ double ld_stream(const double *a, uint64_t pol)
 // ---- nuclide j of material m --------------------------------------------------------------
 struct Row {
     const double *E, *pts, *T;
+    const int32_t *B;
     double conc;
+    int nuc;
 };
 
+// 48 B NucRef as three 16 B broadcast loads (fields a kernel does not use are dead code)
 __device__ __forceinline__ Row load_row(const GridView &gv, int idx)
 {
     const ulonglong2 *p = reinterpret_cast<const ulonglong2 *>(gv.refs + idx);
-    const ulonglong2 a = __ldg(p), b = __ldg(p + 1);
+    const ulonglong2 a = __ldg(p), b = __ldg(p + 1), c = __ldg(p + 2);
     Row r;
     r.E = opaque(reinterpret_cast<const double *>(a.x));
     r.pts = opaque(reinterpret_cast<const double *>(a.y));
     r.T = opaque(reinterpret_cast<const double *>(b.x));
-    r.conc = __longlong_as_double((long long)b.y);
+    r.B = reinterpret_cast<const int32_t *>(b.y);
+    r.conc = __longlong_as_double((long long)c.x);
+    r.nuc = (int)c.y;
+    return r;
+}
+
+// the Row of nuclide `nuc` built from the grid view (debug paths that have no material)
+__device__ __forceinline__ Row make_row(const GridView &gv, int nuc)
+{
+    Row r;
+    r.E = opaque(gv.E + (size_t)nuc * (uint32_t)gv.n);
+    r.pts = gv.pts + (size_t)nuc * (uint32_t)gv.n * 6;
+    r.T = gv.tkeys ? gv.tkeys + (size_t)nuc * (uint32_t)gv.t_per_nuc : nullptr;
+    r.B = gv.bnd ? gv.bnd + (size_t)nuc * (((size_t)1 << gv.b_log2) + 1) : nullptr;
+    r.conc = 0.0;
+    r.nuc = nuc;
     return r;
 }
 
 // ---- the lower index of one (lookup, nuclide) pair ----------------------
 template <int GRID, int SEARCH>
-__device__ __forceinline__ int lower_index(const GridView &gv, const double *__restrict__ Ei, int nuc, double q,
-                                           int e_union)
+__device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, double q, int e_union)
 {
-    if constexpr (GRID == XS_NUCLIDE) {
+    const double *__restrict__ Ei = rw.E;
+    const int nuc = rw.nuc;
+    if constexpr (GRID == XS_NUCLIDE && SEARCH == XS_SEARCH_H) {
+        // bin-bounded window: q * 2^k is exact, so b/2^k <= q < (b+1)/2^k and, L being
+        // monotone, Tb[b] <= L(q) <= Tb[b+1] (<= n-2): Listing 1 on [Tb[b], Tb[b+1]+1]
+        if (gv.b_log2 > 0 && q >= 0.0 && q <= 1.0) {
+            const int nb = 1 << gv.b_log2;
+            int b = (int)__dmul_rn(q, (double)nb);
+            b = b < nb - 1 ? b : nb - 1;
+            const int lo = __ldg(rw.B + b);
+            const int hi = __ldg(rw.B + b + 1) + 1;
+            return search<XS_SEARCH_U2>(Ei, lo, hi, q);
+        }
+        return search<XS_SEARCH_U2>(Ei, 0, gv.n - 1, q);
+    } else if constexpr (GRID == XS_NUCLIDE) {
         return search<SEARCH>(Ei, 0, gv.n - 1, q);
     } else if constexpr (GRID == XS_UNIONIZED) {
         return __ldg(gv.IDX + (size_t)e_union * (uint32_t)gv.n_nuc + nuc);

@@ -96,8 +96,7 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BL
             const int e_union = union_index<GRID, SEARCH>(gv, q);
             for (int jn = 0; jn < nn; jn++) {
                 const Row rw = load_row(gv, row + jn);
-                const int nuc = (GRID == XS_NUCLIDE) ? 0 : __ldg(gv.mats + row + jn);
-                const int L = lower_index<GRID, SEARCH>(gv, rw.E, nuc, q, e_union);
+                const int L = lower_index<GRID, SEARCH>(gv, rw, q, e_union);
                 if (out_idx)
                     out_idx[(size_t)r * gv.max_nucs + jn] = L;
                 accumulate_pair(rw.pts, L, q, rw.conc, A);
@@ -134,7 +133,8 @@ template <int GRID> static FusedFn pick_g(int search, bool sorted, bool outs)
     case XS_SEARCH_M2: return pick_s<GRID, XS_SEARCH_M2>(sorted, outs);
     case XS_SEARCH_M4: return pick_s<GRID, XS_SEARCH_M4>(sorted, outs);
     case XS_SEARCH_M8: return pick_s<GRID, XS_SEARCH_M8>(sorted, outs);
-    default: return pick_s<GRID, XS_SEARCH_W>(sorted, outs);
+    case XS_SEARCH_W: return pick_s<GRID, XS_SEARCH_W>(sorted, outs);
+    default: return pick_s<GRID, XS_SEARCH_H>(sorted, outs);
     }
 }
 

@@ -53,8 +53,7 @@ __global__ void __launch_bounds__(kSearchTpb, 8)
         const int e_union = union_index<GRID, SEARCH>(gv, q);
         for (int jn = 0; jn < nn; jn++) {
             const Row rw = load_row(gv, row + jn);
-            const int nuc = (GRID == XS_NUCLIDE) ? 0 : __ldg(gv.mats + row + jn);
-            dst[(size_t)jn * stride] = lower_index<GRID, SEARCH>(gv, rw.E, nuc, q, e_union);
+            dst[(size_t)jn * stride] = lower_index<GRID, SEARCH>(gv, rw, q, e_union);
         }
     }
 }
@@ -106,7 +105,8 @@ template <int GRID> static SearchKFn pick_g(int search)
     case XS_SEARCH_M2: return k_search<GRID, XS_SEARCH_M2>;
     case XS_SEARCH_M4: return k_search<GRID, XS_SEARCH_M4>;
     case XS_SEARCH_M8: return k_search<GRID, XS_SEARCH_M8>;
-    default: return k_search<GRID, XS_SEARCH_W>;
+    case XS_SEARCH_W: return k_search<GRID, XS_SEARCH_W>;
+    default: return k_search<GRID, XS_SEARCH_H>;
     }
 }
 

@@ -32,7 +32,7 @@ __global__ void k_search_points(GridView gv, int64_t count, const double *__rest
     for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < count; t += (int64_t)gridDim.x * blockDim.x) {
         const double qq = q[t];
         const int nu = nuc[t];
-        out[t] = lower_index<GRID, SEARCH>(gv, nuclide_row(gv, nu), nu, qq, union_index<GRID, SEARCH>(gv, qq));
+        out[t] = lower_index<GRID, SEARCH>(gv, make_row(gv, nu), qq, union_index<GRID, SEARCH>(gv, qq));
     }
 }
 
@@ -50,7 +50,8 @@ template <int GRID> static SearchPtsFn pick_pts(int search)
     case XS_SEARCH_M2: return k_search_points<GRID, XS_SEARCH_M2>;
     case XS_SEARCH_M4: return k_search_points<GRID, XS_SEARCH_M4>;
     case XS_SEARCH_M8: return k_search_points<GRID, XS_SEARCH_M8>;
-    default: return k_search_points<GRID, XS_SEARCH_W>;
+    case XS_SEARCH_W: return k_search_points<GRID, XS_SEARCH_W>;
+    default: return k_search_points<GRID, XS_SEARCH_H>;
     }
 }
 
@@ -157,8 +158,8 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         SortedView so{};
         XS_CUDA_TRY(cudaEventRecord(g.ev[1], stream));
         if (sorted) {
-            launches += launch_bucket_sort(g, sv, nb_log2, !fused, stream);
-            const int K = kMaterials << nb_log2;
+            int K = 0;
+            launches += launch_bucket_sort(g, sv, nb, !fused, stream, &K);
             so.q = g.qs;
             so.q_of = g.sq;
             so.slot = g.si;

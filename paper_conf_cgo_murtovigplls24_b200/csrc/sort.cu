@@ -1,6 +1,7 @@
 // sort.cu -- sampling + the (material, energy) counting sort.
 //
-// Key = (material << nb_log2) | energy bucket, K = 12 << nb_log2 <= 49152 buckets.
+// Key = kbase[material] + energy bucket (BucketPlan: material m gets nb[m] buckets in
+// proportion to P(m) * num_nucs[m], its expected share of the pairs), K <= 49152.
 //   k_bucket_count   sample each lookup of the chunk once (one Listing-7 jump per thread,
 //                    then one affine step per lookup), write its energy and key at its own
 //                    offset (coalesced) and histogram the keys in shared memory
@@ -20,14 +21,22 @@ namespace xs {
 
 constexpr int kSortTpb = 1024;
 
-__global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, int nb_log2, int per_cta, Affine J_tpb,
+__global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
                                                             uint32_t *__restrict__ hist, double *__restrict__ q_of,
                                                             uint16_t *__restrict__ key_of)
 {
     extern __shared__ uint32_t sh[];
-    const int K = kMaterials << nb_log2;
+    __shared__ int s_nb[kMaterials], s_kbase[kMaterials];
+    const int K = bp.K;
     for (int k = threadIdx.x; k < K; k += kSortTpb)
         sh[k] = 0;
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int m = 0; m < kMaterials; m++) {
+            s_nb[m] = bp.nb[m];
+            s_kbase[m] = bp.kbase[m];
+        }
+    }
     __syncthreads();
     const int count = (int)sv.count;
     const int beg = blockIdx.x * per_cta;
@@ -39,7 +48,7 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, int nb
             double q;
             int mat;
             sample_lookup(s, sv, q, mat);
-            const int key = (mat << nb_log2) + energy_bucket(q, nb_log2);
+            const int key = bucket_key(s_nb, s_kbase, mat, q);
             atomicAdd(&sh[key], 1u);
             q_of[j] = q;
             key_of[j] = (uint16_t)key;
@@ -119,10 +128,11 @@ __global__ void k_bucket_colscan(int K, int ctas, uint32_t *hist, uint32_t *__re
 // memory with coalesced loads, each thread scans a contiguous run of ceil(K/1024), a
 // block scan combines the runs, and the results go back coalesced.  Then
 // base[K + m] = first slot of material m (m = 0..11), base[K + 12] = count.
-__global__ void __launch_bounds__(1024) k_bucket_base(int K, int nb_log2, uint32_t *__restrict__ base)
+__global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, uint32_t *__restrict__ base)
 {
     extern __shared__ uint32_t sv[];
     __shared__ uint32_t wsum[32];
+    const int K = bp.K;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     for (int k = threadIdx.x; k < K; k += 1024)
         sv[k] = base[k];
@@ -162,20 +172,22 @@ __global__ void __launch_bounds__(1024) k_bucket_base(int K, int nb_log2, uint32
     __syncthreads();
     for (int k = threadIdx.x; k < K; k += 1024)
         base[k] = sv[k];
-    if (threadIdx.x < kMaterials)
-        base[K + threadIdx.x] = sv[threadIdx.x << nb_log2];
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int m = 0; m < kMaterials; m++)
+            base[K + m] = sv[bp.kbase[m]];
+    }
     if (threadIdx.x == 0)
         base[K + kMaterials] = wsum[31];
 }
 
-__global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int nb_log2, int per_cta, int count,
+__global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int per_cta, int count,
                                                               const uint32_t *__restrict__ hist,
                                                               const uint32_t *__restrict__ base,
                                                               const uint16_t *__restrict__ key_of,
                                                               uint32_t *__restrict__ slot_of)
 {
     extern __shared__ uint32_t sh[];
-    const int K = kMaterials << nb_log2;
     const uint32_t *h = hist + (int64_t)blockIdx.x * K;
     for (int k = threadIdx.x; k < K; k += kSortTpb)
         sh[k] = base[k] + h[k];
@@ -233,7 +245,29 @@ static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
     }
 }
 
-int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gather, cudaStream_t stream)
+static BucketPlan make_plan(const Grid &g, int nb_avg)
+{
+    BucketPlan bp{};
+    double w[kMaterials], W = 0;
+    for (int m = 0; m < kMaterials; m++) {
+        const double p = (m == 0) ? 1.0 - g.thresholds[11] : g.thresholds[m] - g.thresholds[m - 1];
+        w[m] = p * g.num_nucs[m];
+        W += w[m];
+    }
+    // floor(total * share) + at most one bump to 1 per material stays <= 12 * nb_avg
+    const int total = nb_avg > 1 ? kMaterials * (nb_avg - 1) : 0;
+    int k = 0;
+    for (int m = 0; m < kMaterials; m++) {
+        bp.kbase[m] = k;
+        bp.nb[m] = std::max(1, (int)(total * w[m] / W));
+        k += bp.nb[m];
+    }
+    bp.kbase[kMaterials] = k;
+    bp.K = k;
+    return bp;
+}
+
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gather, cudaStream_t stream, int *K_out)
 {
     static bool smem_set[64] = {};
     if (!smem_set[g.device & 63]) {
@@ -244,17 +278,19 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gat
         smem_set[g.device & 63] = true;
     }
     const int64_t cn = sv.count;
-    const int K = kMaterials << nb_log2;
+    const BucketPlan bp = make_plan(g, nb_avg);
+    const int K = bp.K;
+    *K_out = K;
     const int sms = sm_count_dev();
     const int ctas = (int)std::max<int64_t>(1, std::min<int64_t>(sms, (cn + kSortTpb - 1) / kSortTpb));
     const int per_cta = (int)((cn + ctas - 1) / ctas);
     ensure_sort_space(g, cn, ctas, K);
     const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
     const size_t smem = (size_t)K * 4;
-    k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, nb_log2, per_cta, J, g.hist, g.sq, g.skey);
+    k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, bp, per_cta, J, g.hist, g.sq, g.skey);
     k_bucket_colscan<<<(K * kColSplit + 127) / 128, 128, 0, stream>>>(K, ctas, g.hist, g.base);
-    k_bucket_base<<<1, 1024, smem, stream>>>(K, nb_log2, g.base);
-    k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(nb_log2, per_cta, (int)cn, g.hist, g.base, g.skey, g.si);
+    k_bucket_base<<<1, 1024, smem, stream>>>(bp, g.base);
+    k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, per_cta, (int)cn, g.hist, g.base, g.skey, g.si);
     XS_CUDA_TRY(cudaGetLastError());
     if (!with_gather)
         return 4;

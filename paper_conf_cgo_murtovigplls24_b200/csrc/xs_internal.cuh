@@ -64,6 +64,9 @@ struct Grid {
     int32_t t_off[kTreeMaxLevels] = {};
     int32_t t_leaf = 0;       // elements probed at the leaf (<= 16)
     int64_t t_per_nuc = 0;    // keys per nuclide
+    // bin bounds of every nuclide row (XS_SEARCH_H): [n_nuc][2^b_log2 + 1]
+    int32_t *bnd = nullptr;
+    int32_t b_log2 = 0;
     double *U = nullptr;
     int32_t *IDX = nullptr;
     int32_t *H = nullptr;
@@ -114,7 +117,9 @@ struct NucRef {
     const double *E;   // energy row of the nuclide            (E + nuc * n)
     const double *pts; // 48 B point records of the nuclide    (pts + nuc * n * 6)
     const double *T;   // separator tree of the nuclide, or NULL
+    const int32_t *B;  // bin bounds of the nuclide, or NULL
     double conc;       // concs[m][j]
+    int64_t nuc;       // nuclide id
 };
 
 struct GridView {
@@ -139,6 +144,9 @@ struct GridView {
     int32_t t_off[kTreeMaxLevels];
     int32_t t_leaf;
     int32_t t_per_nuc;
+    int32_t b_log2;   // XS_SEARCH_H bins = 2^b_log2 (0: no table)
+    int32_t pad2_;
+    const int32_t *__restrict__ bnd;
 };
 
 struct SampleView {
@@ -172,10 +180,12 @@ void build_grid(Grid &g);
 void free_grid(Grid &g);
 uint64_t grid_checksum(const Grid &g);
 
-// sort.cu: the (material, energy) counting sort of one chunk; leaves g.sq (energy by
-// lookup offset) and g.si (slot -> offset) filled and the material bases at g.base + K
-// (device).  with_gather also fills g.qs (energy by slot).  Returns kernels launched.
-int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_log2, bool with_gather, cudaStream_t stream);
+// sort.cu: the (material, energy) counting sort of one chunk with `nb_avg` energy buckets
+// per material on average; leaves g.sq (energy by lookup offset) and g.si (slot -> offset)
+// filled and the material bases at g.base + *K_out (device).  with_gather also fills g.qs
+// (energy by slot).  Returns the kernels launched.
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gather, cudaStream_t stream,
+                       int *K_out);
 
 // lookup_fused.cu: one kernel per lookup batch (search + interpolation in one thread)
 void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, cudaStream_t stream,

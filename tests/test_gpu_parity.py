@@ -13,7 +13,7 @@ pytestmark = pytest.mark.gpu
 
 from xs_workloads import GRID_SEED, LOOKUP_SEED, WORKLOADS  # noqa: E402
 
-SEARCHES = ["M", "U1", "U2", "U4", "U8", "B", "M2", "M4", "M8", "W"]
+SEARCHES = ["M", "U1", "U2", "U4", "U8", "B", "M2", "M4", "M8", "W", "H"]
 SORTS = ["none", "material", "material_energy"]
 RTOL = 1e-12
 
