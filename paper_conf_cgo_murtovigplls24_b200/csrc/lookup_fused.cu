@@ -14,20 +14,33 @@
 namespace xs {
 
 constexpr int kFusedTpb = 256;
+#ifndef XS_CHUNK_ITERS
+#define XS_CHUNK_ITERS 4
+#endif
+constexpr int kChunkIters = XS_CHUNK_ITERS; // 256-slot iterations per work chunk (sorted)
 #ifndef XS_W_MIN_BLOCKS
 #define XS_W_MIN_BLOCKS 4
+#endif
+#ifndef XS_H_MIN_BLOCKS
+#define XS_H_MIN_BLOCKS 4
 #endif
 
 // OUTS: the call asked for macroscopic XS and/or indices; without it the bench/hash path
 // carries no output pointers (fewer live registers, no spills at 64 per thread)
 template <int GRID, int SEARCH, bool SORTED, bool OUTS>
-__global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BLOCKS : 4)
+__global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W   ? XS_W_MIN_BLOCKS
+                                             : SEARCH == XS_SEARCH_H ? XS_H_MIN_BLOCKS
+                                                                     : 4)
     k_lookup(GridView gv, SampleView sv, SortedView so, Affine J_grid, double *__restrict__ out_,
              int32_t *__restrict__ out_idx_, unsigned long long *__restrict__ stats)
 {
     double *__restrict__ out = OUTS ? out_ : nullptr;
     int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
     constexpr bool kCoop = SORTED && SEARCH == XS_SEARCH_W && GRID == XS_NUCLIDE;
+#ifndef XS_PIPE_H
+#define XS_PIPE_H 1
+#endif
+    constexpr bool kPipeH = XS_PIPE_H && SEARCH == XS_SEARCH_H && GRID == XS_NUCLIDE;
     __shared__ uint32_t s_mb[kMaterials + 1];
     if constexpr (SORTED) {
         if (threadIdx.x <= kMaterials)
@@ -35,10 +48,28 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BL
         __syncthreads();
     }
     uint32_t my_hash = 0, my_pairs = 0;
-    const int count = (int)sv.count;
-    const int G = gridDim.x * blockDim.x;
     const int lane = threadIdx.x & 31;
-    const int j0 = blockIdx.x * blockDim.x + threadIdx.x;
+    const int count = (int)sv.count;
+    // Sorted: a persistent grid pulls chunks of kChunkIters x blockDim consecutive slots
+    // from an atomic counter, in slot order: consecutive iterations of a CTA hit
+    // neighbouring grid intervals (L1 reuse), the whole GPU sweeps the sorted order as one
+    // narrow band (L2 reuse when the grid does not fit), and the load balances itself.
+    // Unsorted: grid-stride over the chunk (XSBench order).
+    __shared__ int s_chunk;
+    const int csize = SORTED ? kChunkIters * (int)blockDim.x : 0;
+    int j0, jend, G;
+    if constexpr (SORTED) {
+        if (threadIdx.x == 0)
+            s_chunk = atomicAdd(so.work, 1);
+        __syncthreads();
+        j0 = s_chunk * csize + threadIdx.x;
+        jend = min(count, s_chunk * csize + csize);
+        G = blockDim.x;
+    } else {
+        j0 = blockIdx.x * blockDim.x + threadIdx.x;
+        jend = count;
+        G = gridDim.x * blockDim.x;
+    }
     uint64_t s = 0;
     uint32_t r_next = 0;
     double q_next = 0.0;
@@ -46,13 +77,19 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BL
     if constexpr (!SORTED) {
         if (j0 < count)
             s = lookup_state(sv, j0);
-    } else if (j0 < count) {
-        r_next = ld_stream(so.slot + j0, pol);
-        q_next = ld_stream(so.q_of + r_next, pol);
     }
-    for (int jw = j0 - lane; jw < count; jw += G) { // warp-uniform trip count
+    for (;;) {
+        if constexpr (SORTED) {
+            if (j0 - (int)threadIdx.x >= count)
+                break;
+            if (j0 < jend) {
+                r_next = ld_stream(so.slot + j0, pol);
+                q_next = ld_stream(so.q_of + r_next, pol);
+            }
+        }
+    for (int jw = j0 - lane; jw < jend; jw += G) { // warp-uniform trip count
         const int j = jw + lane;
-        const bool active = j < count;
+        const bool active = j < jend;
         double q = 0.0;
         int mat = 0;
         uint32_t r = 0;
@@ -62,7 +99,7 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BL
                 // dependent random 8 B read of q_of overlaps a whole lookup's searches
                 q = q_next;
                 r = r_next;
-                if (j + G < count) {
+                if (j + G < jend) {
                     r_next = ld_stream(so.slot + j + G, pol);
                     q_next = ld_stream(so.q_of + r_next, pol);
                 }
@@ -92,6 +129,33 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BL
                     out_idx[(size_t)r * gv.max_nucs + jn] = L;
                 accumulate_pair(rw.pts, L, q, rw.conc, A);
             }
+        } else if (kPipeH && active) {
+            // bin-bounded search, software-pipelined: the next nuclide's row and window
+            // bounds (independent of this nuclide) are loaded while this one is searched,
+            // gathered and interpolated
+            const bool in01 = q >= 0.0 && q <= 1.0 && gv.b_log2 > 0;
+            const int nbins = 1 << gv.b_log2;
+            int bq = in01 ? (int)__dmul_rn(q, (double)nbins) : 0;
+            bq = bq < nbins - 1 ? bq : nbins - 1;
+            Row rw = load_row(gv, row);
+            int lo = in01 ? __ldg(rw.B + bq) : 0;
+            int hi = in01 ? __ldg(rw.B + bq + 1) + 1 : gv.n - 1;
+            for (int jn = 0; jn < nn; jn++) {
+                Row rn = rw;
+                int lo_n = 0, hi_n = 0;
+                if (jn + 1 < nn) {
+                    rn = load_row(gv, row + jn + 1);
+                    lo_n = in01 ? __ldg(rn.B + bq) : 0;
+                    hi_n = in01 ? __ldg(rn.B + bq + 1) + 1 : gv.n - 1;
+                }
+                const int L = search<XS_SEARCH_U2>(rw.E, lo, hi, q);
+                if (out_idx)
+                    out_idx[(size_t)r * gv.max_nucs + jn] = L;
+                accumulate_pair(rw.pts, L, q, rw.conc, A);
+                rw = rn;
+                lo = lo_n;
+                hi = hi_n;
+            }
         } else if (active) {
             const int e_union = union_index<GRID, SEARCH>(gv, q);
             for (int jn = 0; jn < nn; jn++) {
@@ -107,6 +171,17 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W ? XS_W_MIN_BL
             my_pairs += (uint32_t)nn;
             if (out)
                 store_macro(out, r, A);
+        }
+    }
+        if constexpr (!SORTED)
+            break;
+        else { // next chunk
+            __syncthreads();
+            if (threadIdx.x == 0)
+                s_chunk = atomicAdd(so.work, 1);
+            __syncthreads();
+            j0 = s_chunk * csize + threadIdx.x;
+            jend = min(count, s_chunk * csize + csize);
         }
     }
     reduce_stats<kFusedTpb>(my_hash, my_pairs, stats);

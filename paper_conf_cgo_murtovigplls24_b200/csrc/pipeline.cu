@@ -164,6 +164,8 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             so.q_of = g.sq;
             so.slot = g.si;
             so.mb_dev = g.base + K;
+            so.work = reinterpret_cast<int *>(g.stats_d + 4);
+            XS_CUDA_TRY(cudaMemsetAsync(so.work, 0, sizeof(int), stream));
             if (!fused) {
                 XS_CUDA_TRY(cudaMemcpyAsync(g.mb_h, g.base + K, (kMaterials + 1) * sizeof(uint32_t),
                                             cudaMemcpyDeviceToHost, stream));
@@ -175,7 +177,9 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         XS_CUDA_TRY(cudaEventRecord(g.ev[2], stream));
         XS_CUDA_TRY(cudaEventRecord(g.ev[3], stream));
         if (fused) {
-            const int blocks = blocks_for(cn, tpb, (2048 / tpb) * 4);
+            // sorted: a persistent grid (one resident wave) pulling work chunks;
+            // unsorted: 4 waves of grid-stride CTAs
+            const int blocks = blocks_for(cn, tpb, sorted ? (1024 / tpb) : (2048 / tpb) * 4);
             const Affine Jg = lcg_jump(2 * (uint64_t)blocks * tpb);
             launch_fused(g.grid_type, o.search, sorted, blocks, tpb, stream, gv, sv, so, Jg, outp, idxp, stats);
             launches += 1;

@@ -62,123 +62,116 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, Bucket
 }
 
 // per bucket k: exclusive scan over the CTAs, in place; total[k] = the bucket's size.
-// 4 threads per bucket (adjacent lanes) each own a quarter of the CTA rows, so the
-// dependent chain of row loads is 4x shorter; loads are batched by 8.
-constexpr int kColSplit = 4;
+// A CTA owns 32 buckets (lane = bucket, one coalesced 128 B row segment per load) and its 8
+// warps own 1/8 of the CTA rows each, so every lane keeps ~19 independent loads in flight;
+// the 8 warp partials per bucket are scanned through shared memory.
+constexpr int kColWarps = 8;
 
-__device__ __forceinline__ uint32_t colsum(const uint32_t *hist, int K, int k, int c0, int c1)
+__global__ void __launch_bounds__(32 * kColWarps) k_bucket_colscan(int K, int ctas, uint32_t *hist,
+                                                                    uint32_t *__restrict__ total)
 {
-    uint32_t run = 0;
-    int c = c0;
-    for (; c + 8 <= c1; c += 8) {
-        uint32_t v[8];
+    __shared__ uint32_t part[kColWarps][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int k = blockIdx.x * 32 + lane;
+    const int per = (ctas + kColWarps - 1) / kColWarps;
+    const int c0 = min(w * per, ctas), c1 = min(c0 + per, ctas);
+    // rows are held in registers between the two passes (<= 32 per warp: ctas <= 256;
+    // larger row counts take the slow path below)
+    constexpr int kMaxRows = 32;
+    uint32_t v[kMaxRows];
+    uint32_t sum = 0;
+    const bool fast = (c1 - c0) <= kMaxRows;
+    if (k < K) {
+        if (fast) {
 #pragma unroll
-        for (int u = 0; u < 8; u++)
-            v[u] = hist[(int64_t)(c + u) * K + k];
+            for (int u = 0; u < kMaxRows; u++)
+                v[u] = (c0 + u < c1) ? hist[(int64_t)(c0 + u) * K + k] : 0u;
 #pragma unroll
-        for (int u = 0; u < 8; u++)
-            run += v[u];
-    }
-    for (; c < c1; c++)
-        run += hist[(int64_t)c * K + k];
-    return run;
-}
-
-__global__ void k_bucket_colscan(int K, int ctas, uint32_t *hist, uint32_t *__restrict__ total)
-{
-    const int tid = blockIdx.x * blockDim.x + threadIdx.x;
-    const int k = tid / kColSplit, part = tid % kColSplit;
-    const int per = (ctas + kColSplit - 1) / kColSplit;
-    const int c0 = min(part * per, ctas), c1 = min(c0 + per, ctas);
-    const bool valid = k < K;
-    const uint32_t mine = valid ? colsum(hist, K, k, c0, c1) : 0u;
-    // exclusive scan of the 4 partial sums (lanes 4k'..4k'+3 of the warp)
-    uint32_t incl = mine;
-#pragma unroll
-    for (int o = 1; o < kColSplit; o <<= 1) {
-        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o, kColSplit);
-        if (part >= o)
-            incl += t;
-    }
-    if (!valid)
-        return;
-    uint32_t run = incl - mine;
-    int c = c0;
-    for (; c + 8 <= c1; c += 8) {
-        uint32_t v[8];
-#pragma unroll
-        for (int u = 0; u < 8; u++)
-            v[u] = hist[(int64_t)(c + u) * K + k];
-#pragma unroll
-        for (int u = 0; u < 8; u++) {
-            hist[(int64_t)(c + u) * K + k] = run;
-            run += v[u];
+            for (int u = 0; u < kMaxRows; u++)
+                sum += v[u];
+        } else {
+            for (int c = c0; c < c1; c++)
+                sum += hist[(int64_t)c * K + k];
         }
     }
-    for (; c < c1; c++) {
-        const uint32_t v = hist[(int64_t)c * K + k];
-        hist[(int64_t)c * K + k] = run;
-        run += v;
+    part[w][lane] = sum;
+    __syncthreads();
+    uint32_t off = 0;
+    for (int v = 0; v < w; v++)
+        off += part[v][lane];
+    if (w == kColWarps - 1 && k < K)
+        total[k] = off + sum;
+    if (k < K) {
+        if (fast) {
+#pragma unroll
+            for (int u = 0; u < kMaxRows; u++)
+                if (c0 + u < c1) {
+                    hist[(int64_t)(c0 + u) * K + k] = off;
+                    off += v[u];
+                }
+        } else {
+            for (int c = c0; c < c1; c++) {
+                const uint32_t x = hist[(int64_t)c * K + k];
+                hist[(int64_t)c * K + k] = off;
+                off += x;
+            }
+        }
     }
-    if (part == kColSplit - 1)
-        total[k] = run;
 }
 
-// one CTA: exclusive scan of base[0..K) in place.  All K values are staged in shared
-// memory with coalesced loads, each thread scans a contiguous run of ceil(K/1024), a
-// block scan combines the runs, and the results go back coalesced.  Then
-// base[K + m] = first slot of material m (m = 0..11), base[K + 12] = count.
+// one CTA: exclusive scan of base[0..K) in place.  Warp w owns a contiguous segment and
+// walks it 32 coalesced elements at a time (warp scan + carry) -- no bank conflicts;
+// a block scan of the warp totals gives each warp its offset for the second pass.  Then
+// base[K + m] = first slot of material m, base[K + 12] = count.
 __global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, uint32_t *__restrict__ base)
 {
-    extern __shared__ uint32_t sv[];
     __shared__ uint32_t wsum[32];
     const int K = bp.K;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (int k = threadIdx.x; k < K; k += 1024)
-        sv[k] = base[k];
-    __syncthreads();
-    const int per = (K + 1023) / 1024;
-    const int b0 = min((int)threadIdx.x * per, K), b1 = min(b0 + per, K);
-    uint32_t mine = 0;
-    for (int k = b0; k < b1; k++)
-        mine += sv[k];
-    uint32_t incl = mine;
+    const int seg = ((K + 31) / 32 + 31) / 32 * 32; // elements per warp, multiple of 32
+    const int b0 = min(wid * seg, K), b1 = min(b0 + seg, K);
+    uint32_t tot = 0;
+    for (int k = b0 + lane; k < b1; k += 32)
+        tot += base[k];
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o)
-            incl += t;
-    }
-    if (lane == 31)
-        wsum[wid] = incl;
+    for (int o = 16; o > 0; o >>= 1)
+        tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    if (lane == 0)
+        wsum[wid] = tot;
     __syncthreads();
     if (wid == 0) {
-        uint32_t w = wsum[lane];
+        uint32_t v = wsum[lane];
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t t = __shfl_up_sync(0xffffffffu, w, o);
+            const uint32_t t = __shfl_up_sync(0xffffffffu, v, o);
             if (lane >= o)
-                w += t;
+                v += t;
         }
-        wsum[lane] = w;
+        wsum[lane] = v; // inclusive
     }
     __syncthreads();
-    uint32_t run = incl - mine + (wid ? wsum[wid - 1] : 0u);
-    for (int k = b0; k < b1; k++) {
-        const uint32_t v = sv[k];
-        sv[k] = run;
-        run += v;
+    uint32_t carry = wid ? wsum[wid - 1] : 0u;
+    for (int r = b0; r < b1; r += 32) {
+        const int k = r + lane;
+        const uint32_t v = k < b1 ? base[k] : 0u;
+        uint32_t incl = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o)
+                incl += t;
+        }
+        if (k < b1)
+            base[k] = carry + incl - v;
+        carry += __shfl_sync(0xffffffffu, incl, 31);
     }
     __syncthreads();
-    for (int k = threadIdx.x; k < K; k += 1024)
-        base[k] = sv[k];
     if (threadIdx.x == 0) {
 #pragma unroll
         for (int m = 0; m < kMaterials; m++)
-            base[K + m] = sv[bp.kbase[m]];
-    }
-    if (threadIdx.x == 0)
+            base[K + m] = base[bp.kbase[m]];
         base[K + kMaterials] = wsum[31];
+    }
 }
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int per_cta, int count,
@@ -194,9 +187,20 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int per_cta,
     __syncthreads();
     const int beg = blockIdx.x * per_cta;
     const int end = min(beg + per_cta, count);
-    // (recording each lookup's rank in the count pass to drop these atomics was measured
-    // slower: the scatter is bound by its random 4 B stores, not by the atomics)
-    for (int j = beg + threadIdx.x; j < end; j += kSortTpb)
+    // 4 keys in flight per thread, then their shared-memory atomics and 4 B stores
+    // (recording each lookup's rank in the count pass to drop the atomics was measured
+    // slower)
+    int j = beg + threadIdx.x;
+    for (; j + 3 * kSortTpb < end; j += 4 * kSortTpb) {
+        uint32_t kk[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++)
+            kk[u] = key_of[j + u * kSortTpb];
+#pragma unroll
+        for (int u = 0; u < 4; u++)
+            slot_of[atomicAdd(&sh[kk[u]], 1u)] = (uint32_t)(j + u * kSortTpb);
+    }
+    for (; j < end; j += kSortTpb)
         slot_of[atomicAdd(&sh[key_of[j]], 1u)] = (uint32_t)j;
 }
 
@@ -274,7 +278,6 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gath
         const int bytes = kMaterials * kMaxEnergyBins * 4;
         XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_count, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
         XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
-        XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_base, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
         smem_set[g.device & 63] = true;
     }
     const int64_t cn = sv.count;
@@ -288,8 +291,8 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gath
     const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
     const size_t smem = (size_t)K * 4;
     k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, bp, per_cta, J, g.hist, g.sq, g.skey);
-    k_bucket_colscan<<<(K * kColSplit + 127) / 128, 128, 0, stream>>>(K, ctas, g.hist, g.base);
-    k_bucket_base<<<1, 1024, smem, stream>>>(bp, g.base);
+    k_bucket_colscan<<<(K + 31) / 32, 32 * kColWarps, 0, stream>>>(K, ctas, g.hist, g.base);
+    k_bucket_base<<<1, 1024, 0, stream>>>(bp, g.base);
     k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, per_cta, (int)cn, g.hist, g.base, g.skey, g.si);
     XS_CUDA_TRY(cudaGetLastError());
     if (!with_gather)

@@ -76,7 +76,7 @@ struct Grid {
     void *refs = nullptr;            // NucRef [12][max_nucs]: row pointers + conc per (mat, j)
 
     // per-grid scratch (grown on demand; calls on one grid are serialised by the caller)
-    uint64_t *stats_d = nullptr;     // [4] hash, pairs
+    uint64_t *stats_d = nullptr;     // [8] hash, pairs, work counter
     uint64_t *stats_h = nullptr;     // pinned mirror
     double *sq = nullptr;            // energies by lookup offset (coalesced writes) [cap]
     uint32_t *si = nullptr;          // lookup offsets in (material, energy) order  [cap]
@@ -165,6 +165,7 @@ struct SortedView {
     const double *__restrict__ q_of;     // energy by lookup offset
     const uint32_t *__restrict__ slot;   // lookup offset (i - first) of sorted slot j
     const uint32_t *__restrict__ mb_dev; // device copy of matbase (fused path)
+    int *work;                           // fused path: work-chunk counter (zeroed per chunk)
     uint32_t matbase[kMaterials + 1];    // split path: first slot of each material; [12] = count
 };
 
