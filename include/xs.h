@@ -69,8 +69,9 @@ enum {
                          2^k >= n_gridpoints (built at grid creation); q*2^k is exact, so
                          L(q) lies in [Tb[b], Tb[b+1]] for b = floor(q*2^k) and Listing 1
                          (U2) runs on that window -- usually 1-2 points.  XSBench's hash-
-                         grid idea (R7) at power-of-two resolution.  Nuclide grid only;
-                         elsewhere it is U2.                                              */
+                         grid idea (R7) at power-of-two resolution.  On the unionized grid
+                         the same table over U bounds the one U search per lookup; on the
+                         hash grid (whose 10,000-bin table is the configuration) it is U2. */
     XS_SEARCH_COUNT = 11
 };
 

@@ -309,6 +309,17 @@ void build_grid(Grid &g)
             XS_CUDA_TRY(cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, g.E, g.U, (int)N));
             XS_CUDA_TRY(cudaMalloc(&tmp, tmp_bytes));
             XS_CUDA_TRY(cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, g.E, g.U, (int)N));
+            // bin bounds of U (XS_SEARCH_H): UB[b] = Listing1(U, b / 2^k), 2^k >= N
+            {
+                int u_log2 = 1;
+                while ((int64_t(1) << u_log2) < N && u_log2 < 26)
+                    u_log2++;
+                g.u_log2 = u_log2;
+                g.ubnd = dalloc<int32_t>(g, (int64_t(1) << u_log2) + 1);
+                k_bounds_build<<<grid_blocks((int64_t(1) << u_log2) + 1, tpb), tpb>>>(1, (int32_t)N, u_log2, g.U,
+                                                                                       g.ubnd);
+                XS_CUDA_TRY(cudaGetLastError());
+            }
             g.IDX = dalloc<int32_t>(g, N * g.n_nuc);
             const int64_t total = N * g.n_nuc;
             k_union_idx<<<grid_blocks(total, tpb), tpb>>>(total, (int32_t)g.n_nuc, n, g.E, g.U, g.IDX);
@@ -368,6 +379,7 @@ void free_grid(Grid &g)
     cudaFree(g.pts);
     cudaFree(g.tkeys);
     cudaFree(g.bnd);
+    cudaFree(g.ubnd);
     cudaFree(g.U);
     cudaFree(g.IDX);
     cudaFree(g.H);
@@ -456,6 +468,8 @@ GridView make_view(const Grid &g)
     v.t_per_nuc = (int32_t)g.t_per_nuc;
     v.b_log2 = g.bnd ? g.b_log2 : 0;
     v.bnd = g.bnd;
+    v.u_log2 = g.ubnd ? g.u_log2 : 0;
+    v.ubnd = g.ubnd;
     return v;
 }
 

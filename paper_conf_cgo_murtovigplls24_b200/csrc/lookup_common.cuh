@@ -149,10 +149,20 @@ __device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, do
 template <int GRID, int SEARCH>
 __device__ __forceinline__ int union_index(const GridView &gv, double q)
 {
-    if constexpr (GRID == XS_UNIONIZED)
+    if constexpr (GRID == XS_UNIONIZED && SEARCH == XS_SEARCH_H) {
+        // the same bin-bounded window over the unionized energies (R4 + §6.5)
+        if (gv.u_log2 > 0 && q >= 0.0 && q <= 1.0) {
+            const int nb = 1 << gv.u_log2;
+            int b = (int)__dmul_rn(q, (double)nb);
+            b = b < nb - 1 ? b : nb - 1;
+            return search<XS_SEARCH_U2>(opaque(gv.U), __ldg(gv.ubnd + b), __ldg(gv.ubnd + b + 1) + 1, q);
+        }
+        return search<XS_SEARCH_U2>(opaque(gv.U), 0, gv.N - 1, q);
+    } else if constexpr (GRID == XS_UNIONIZED) {
         return search<SEARCH>(opaque(gv.U), 0, gv.N - 1, q);
-    else
+    } else {
         return 0;
+    }
 }
 
 __device__ __forceinline__ const double *nuclide_row(const GridView &gv, int nuc)

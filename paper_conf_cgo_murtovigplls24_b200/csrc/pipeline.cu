@@ -100,6 +100,9 @@ template <class T> static void grow(T *&p, int64_t &cap, int64_t need)
 }
 
 constexpr int64_t kChunkFused = int64_t(1) << 28;  // uint32 slots
+// one sort per 2^28 lookups: a 2^25 cap kept the 4 B slot array L2-sized and halved the
+// sort time of 100M lookups, but the coarser ordering cost more in the lookup kernel
+constexpr int64_t kChunkSorted = int64_t(1) << 28;
 constexpr int64_t kChunkSplit = int64_t(1) << 25;  // pair buffer <= 33.5M x 321 x 4 B
 constexpr int64_t kChunkHost = int64_t(1) << 22;   // staging for host outputs (x2 buffers)
 
@@ -118,9 +121,13 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
     const bool sorted = o.sort != XS_SORT_NONE;
     const bool fused = !sorted || !(o.flags & XS_FLAG_SPLIT);
     const bool host_out = out_macro && !is_device_accessible(out_macro);
-    int64_t chunk = fused ? kChunkFused : kChunkSplit;
+    int64_t chunk = fused ? (sorted ? kChunkSorted : kChunkFused) : kChunkSplit;
     if (host_out)
         chunk = std::min(chunk, kChunkHost);
+    if (count > chunk) { // equal chunks (no small tail chunk)
+        const int64_t nch = (count + chunk - 1) / chunk;
+        chunk = (count + nch - 1) / nch;
+    }
     const GridView gv = make_view(g);
     int launches = 0;
     double sample_ms = 0, lookup_ms = 0, search_ms = 0, copy_ms = 0;

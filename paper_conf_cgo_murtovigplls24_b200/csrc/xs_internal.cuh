@@ -67,6 +67,9 @@ struct Grid {
     // bin bounds of every nuclide row (XS_SEARCH_H): [n_nuc][2^b_log2 + 1]
     int32_t *bnd = nullptr;
     int32_t b_log2 = 0;
+    // bin bounds of the unionized energies (XS_SEARCH_H on XS_UNIONIZED): [2^u_log2 + 1]
+    int32_t *ubnd = nullptr;
+    int32_t u_log2 = 0;
     double *U = nullptr;
     int32_t *IDX = nullptr;
     int32_t *H = nullptr;
@@ -145,8 +148,9 @@ struct GridView {
     int32_t t_leaf;
     int32_t t_per_nuc;
     int32_t b_log2;   // XS_SEARCH_H bins = 2^b_log2 (0: no table)
-    int32_t pad2_;
+    int32_t u_log2;   // unionized XS_SEARCH_H bins = 2^u_log2 (0: no table)
     const int32_t *__restrict__ bnd;
+    const int32_t *__restrict__ ubnd;
 };
 
 struct SampleView {
