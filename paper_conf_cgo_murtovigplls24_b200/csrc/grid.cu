@@ -158,17 +158,25 @@ __global__ void k_tree_build(int64_t n_nuc, int32_t n, int32_t levels, int4 stri
     }
 }
 
-// bin bounds: B[nuc][b] = L_nuc(b / 2^b_log2), b = 0 .. 2^b_log2 (the energy is exact)
-__global__ void k_bounds_build(int64_t n_nuc, int32_t n, int32_t b_log2, const double *__restrict__ E,
-                               int32_t *__restrict__ B)
+// bin table: entry (nuc, b) = {L(b/2^k), L((b+1)/2^k) - L(b/2^k), E[L(b/2^k) + 1]} of the
+// row (the energies b/2^k are exact in fp64)
+__global__ void k_bins_build(int64_t n_nuc, int32_t n, int32_t b_log2, const double *__restrict__ E,
+                             BinEntry *__restrict__ B)
 {
-    const int64_t per = ((int64_t)1 << b_log2) + 1;
+    const int64_t per = (int64_t)1 << b_log2;
     const int64_t total = n_nuc * per;
-    const double scale = 1.0 / (double)((int64_t)1 << b_log2);
+    const double scale = 1.0 / (double)per;
     for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < total; g += (int64_t)gridDim.x * blockDim.x) {
         const int64_t nuc = g / per;
         const int64_t b = g - nuc * per;
-        B[g] = search_M<1>(E + nuc * n, 0, n - 1, __dmul_rn((double)b, scale));
+        const double *row = E + nuc * n;
+        const int lo = search_M<1>(row, 0, n - 1, __dmul_rn((double)b, scale));
+        const int hi = search_M<1>(row, 0, n - 1, __dmul_rn((double)(b + 1), scale));
+        BinEntry e;
+        e.lo = lo;
+        e.cnt = hi - lo;
+        e.e_next = row[lo + 1 < n ? lo + 1 : n - 1];
+        B[g] = e;
     }
 }
 
@@ -294,11 +302,11 @@ void build_grid(Grid &g)
             int b_log2 = 1;
             while ((int64_t(1) << b_log2) < g.n && b_log2 < 20)
                 b_log2++;
-            const int64_t per = (int64_t(1) << b_log2) + 1;
+            const int64_t per = int64_t(1) << b_log2;
             if (g.n_nuc * per < (int64_t(1) << 31)) {
                 g.b_log2 = b_log2;
-                g.bnd = dalloc<int32_t>(g, g.n_nuc * per);
-                k_bounds_build<<<grid_blocks(g.n_nuc * per, tpb), tpb>>>(g.n_nuc, n, b_log2, g.E, g.bnd);
+                g.bnd = dalloc<BinEntry>(g, g.n_nuc * per);
+                k_bins_build<<<grid_blocks(g.n_nuc * per, tpb), tpb>>>(g.n_nuc, n, b_log2, g.E, g.bnd);
                 XS_CUDA_TRY(cudaGetLastError());
             }
         }
@@ -315,9 +323,8 @@ void build_grid(Grid &g)
                 while ((int64_t(1) << u_log2) < N && u_log2 < 26)
                     u_log2++;
                 g.u_log2 = u_log2;
-                g.ubnd = dalloc<int32_t>(g, (int64_t(1) << u_log2) + 1);
-                k_bounds_build<<<grid_blocks((int64_t(1) << u_log2) + 1, tpb), tpb>>>(1, (int32_t)N, u_log2, g.U,
-                                                                                       g.ubnd);
+                g.ubnd = dalloc<BinEntry>(g, int64_t(1) << u_log2);
+                k_bins_build<<<grid_blocks(int64_t(1) << u_log2, tpb), tpb>>>(1, (int32_t)N, u_log2, g.U, g.ubnd);
                 XS_CUDA_TRY(cudaGetLastError());
             }
             g.IDX = dalloc<int32_t>(g, N * g.n_nuc);
@@ -352,6 +359,7 @@ void build_grid(Grid &g)
     XS_CUDA_TRY(cudaMemcpy(g.num_nucs_d, g.num_nucs, 12 * sizeof(int32_t), cudaMemcpyHostToDevice));
     {
         std::vector<NucRef> refs((size_t)12 * g.max_nucs, NucRef{nullptr, nullptr, nullptr, nullptr, 0.0, 0});
+        static_assert(sizeof(NucRef) == 48, "NucRef is loaded as three 16 B vectors");
         for (int m = 0; m < 12; m++)
             for (int j = 0; j < g.num_nucs[m]; j++) {
                 const int64_t nuc = mats[(size_t)m * g.max_nucs + j];
@@ -359,7 +367,7 @@ void build_grid(Grid &g)
                 r.E = g.E + nuc * g.n;
                 r.pts = g.pts + nuc * g.n * 6;
                 r.T = g.tkeys ? g.tkeys + nuc * g.t_per_nuc : nullptr;
-                r.B = g.bnd ? g.bnd + nuc * ((int64_t(1) << g.b_log2) + 1) : nullptr;
+                r.B = g.bnd ? g.bnd + nuc * (int64_t(1) << g.b_log2) : nullptr;
                 r.conc = concs[(size_t)m * g.max_nucs + j];
                 r.nuc = nuc;
             }

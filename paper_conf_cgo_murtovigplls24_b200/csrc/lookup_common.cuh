@@ -80,10 +80,38 @@ __device__ __forceinline__ double ld_stream(const double *a, uint64_t pol)
 // ---- nuclide j of material m --------------------------------------------------------------
 struct Row {
     const double *E, *pts, *T;
-    const int32_t *B;
+    const BinEntry *B;
     double conc;
     int nuc;
 };
+
+struct Bin {
+    int lo, cnt;
+    double e_next;
+};
+
+__device__ __forceinline__ Bin load_bin(const BinEntry *p)
+{
+    const int4 v = __ldg(reinterpret_cast<const int4 *>(p));
+    return Bin{v.x, v.y, __hiloint2double(v.w, v.z)};
+}
+
+// the bin of q: q * 2^k is exact, so b/2^k <= q < (b+1)/2^k (q = 1.0 -> last bin)
+__device__ __forceinline__ int bin_of(double q, int log2_bins)
+{
+    const int nb = 1 << log2_bins;
+    const int b = (int)__dmul_rn(q, (double)nb);
+    return b < nb - 1 ? b : nb - 1;
+}
+
+// L(q) from its bin: no row access when the bin holds <= 1 point, else Listing 1 on the
+// bin's window [lo, lo + cnt + 1] (L monotone: lo <= L(q) <= lo + cnt <= n-2)
+__device__ __forceinline__ int bin_lower(const double *__restrict__ A, const Bin &bn, double q)
+{
+    if (bn.cnt <= 1)
+        return bn.lo + ((bn.cnt == 1 && bn.e_next <= q) ? 1 : 0);
+    return search<XS_SEARCH_U2>(A, bn.lo, bn.lo + bn.cnt + 1, q);
+}
 
 // 48 B NucRef as three 16 B broadcast loads (fields a kernel does not use are dead code)
 __device__ __forceinline__ Row load_row(const GridView &gv, int idx)
@@ -94,7 +122,7 @@ __device__ __forceinline__ Row load_row(const GridView &gv, int idx)
     r.E = opaque(reinterpret_cast<const double *>(a.x));
     r.pts = opaque(reinterpret_cast<const double *>(a.y));
     r.T = opaque(reinterpret_cast<const double *>(b.x));
-    r.B = reinterpret_cast<const int32_t *>(b.y);
+    r.B = reinterpret_cast<const BinEntry *>(b.y);
     r.conc = __longlong_as_double((long long)c.x);
     r.nuc = (int)c.y;
     return r;
@@ -107,7 +135,7 @@ __device__ __forceinline__ Row make_row(const GridView &gv, int nuc)
     r.E = opaque(gv.E + (size_t)nuc * (uint32_t)gv.n);
     r.pts = gv.pts + (size_t)nuc * (uint32_t)gv.n * 6;
     r.T = gv.tkeys ? gv.tkeys + (size_t)nuc * (uint32_t)gv.t_per_nuc : nullptr;
-    r.B = gv.bnd ? gv.bnd + (size_t)nuc * (((size_t)1 << gv.b_log2) + 1) : nullptr;
+    r.B = gv.bnd ? gv.bnd + ((size_t)nuc << gv.b_log2) : nullptr;
     r.conc = 0.0;
     r.nuc = nuc;
     return r;
@@ -120,16 +148,9 @@ __device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, do
     const double *__restrict__ Ei = rw.E;
     const int nuc = rw.nuc;
     if constexpr (GRID == XS_NUCLIDE && SEARCH == XS_SEARCH_H) {
-        // bin-bounded window: q * 2^k is exact, so b/2^k <= q < (b+1)/2^k and, L being
-        // monotone, Tb[b] <= L(q) <= Tb[b+1] (<= n-2): Listing 1 on [Tb[b], Tb[b+1]+1]
-        if (gv.b_log2 > 0 && q >= 0.0 && q <= 1.0) {
-            const int nb = 1 << gv.b_log2;
-            int b = (int)__dmul_rn(q, (double)nb);
-            b = b < nb - 1 ? b : nb - 1;
-            const int lo = __ldg(rw.B + b);
-            const int hi = __ldg(rw.B + b + 1) + 1;
-            return search<XS_SEARCH_U2>(Ei, lo, hi, q);
-        }
+        // bin-bounded window
+        if (gv.b_log2 > 0 && q >= 0.0 && q <= 1.0)
+            return bin_lower(Ei, load_bin(rw.B + bin_of(q, gv.b_log2)), q);
         return search<XS_SEARCH_U2>(Ei, 0, gv.n - 1, q);
     } else if constexpr (GRID == XS_NUCLIDE) {
         return search<SEARCH>(Ei, 0, gv.n - 1, q);
@@ -151,12 +172,8 @@ __device__ __forceinline__ int union_index(const GridView &gv, double q)
 {
     if constexpr (GRID == XS_UNIONIZED && SEARCH == XS_SEARCH_H) {
         // the same bin-bounded window over the unionized energies (R4 + §6.5)
-        if (gv.u_log2 > 0 && q >= 0.0 && q <= 1.0) {
-            const int nb = 1 << gv.u_log2;
-            int b = (int)__dmul_rn(q, (double)nb);
-            b = b < nb - 1 ? b : nb - 1;
-            return search<XS_SEARCH_U2>(opaque(gv.U), __ldg(gv.ubnd + b), __ldg(gv.ubnd + b + 1) + 1, q);
-        }
+        if (gv.u_log2 > 0 && q >= 0.0 && q <= 1.0)
+            return bin_lower(opaque(gv.U), load_bin(gv.ubnd + bin_of(q, gv.u_log2)), q);
         return search<XS_SEARCH_U2>(opaque(gv.U), 0, gv.N - 1, q);
     } else if constexpr (GRID == XS_UNIONIZED) {
         return search<SEARCH>(opaque(gv.U), 0, gv.N - 1, q);

@@ -37,8 +37,8 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W   ? XS_W_MIN_
     double *__restrict__ out = OUTS ? out_ : nullptr;
     int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
     constexpr bool kCoop = SORTED && SEARCH == XS_SEARCH_W && GRID == XS_NUCLIDE;
-#ifndef XS_PIPE_H
-#define XS_PIPE_H 1
+#ifndef XS_PIPE_H // software-pipelined H path: measured slower (register spills) -> off
+#define XS_PIPE_H 0
 #endif
     constexpr bool kPipeH = XS_PIPE_H && SEARCH == XS_SEARCH_H && GRID == XS_NUCLIDE;
     __shared__ uint32_t s_mb[kMaterials + 1];
@@ -130,31 +130,27 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W   ? XS_W_MIN_
                 accumulate_pair(rw.pts, L, q, rw.conc, A);
             }
         } else if (kPipeH && active) {
-            // bin-bounded search, software-pipelined: the next nuclide's row and window
-            // bounds (independent of this nuclide) are loaded while this one is searched,
-            // gathered and interpolated
+            // bin-bounded search, software-pipelined: the next nuclide's row and bin entry
+            // (independent of this nuclide) load while this one is resolved, gathered and
+            // interpolated
             const bool in01 = q >= 0.0 && q <= 1.0 && gv.b_log2 > 0;
-            const int nbins = 1 << gv.b_log2;
-            int bq = in01 ? (int)__dmul_rn(q, (double)nbins) : 0;
-            bq = bq < nbins - 1 ? bq : nbins - 1;
+            const int bq = in01 ? bin_of(q, gv.b_log2) : 0;
+            const Bin full{0, gv.n - 2, 0.0}; // window [0, n-1]: the full search
             Row rw = load_row(gv, row);
-            int lo = in01 ? __ldg(rw.B + bq) : 0;
-            int hi = in01 ? __ldg(rw.B + bq + 1) + 1 : gv.n - 1;
+            Bin bn = in01 ? load_bin(rw.B + bq) : full;
             for (int jn = 0; jn < nn; jn++) {
                 Row rn = rw;
-                int lo_n = 0, hi_n = 0;
+                Bin bn_n = bn;
                 if (jn + 1 < nn) {
                     rn = load_row(gv, row + jn + 1);
-                    lo_n = in01 ? __ldg(rn.B + bq) : 0;
-                    hi_n = in01 ? __ldg(rn.B + bq + 1) + 1 : gv.n - 1;
+                    bn_n = in01 ? load_bin(rn.B + bq) : full;
                 }
-                const int L = search<XS_SEARCH_U2>(rw.E, lo, hi, q);
+                const int L = bin_lower(rw.E, bn, q);
                 if (out_idx)
                     out_idx[(size_t)r * gv.max_nucs + jn] = L;
                 accumulate_pair(rw.pts, L, q, rw.conc, A);
                 rw = rn;
-                lo = lo_n;
-                hi = hi_n;
+                bn = bn_n;
             }
         } else if (active) {
             const int e_union = union_index<GRID, SEARCH>(gv, q);

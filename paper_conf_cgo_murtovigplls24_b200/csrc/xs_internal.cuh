@@ -64,11 +64,11 @@ struct Grid {
     int32_t t_off[kTreeMaxLevels] = {};
     int32_t t_leaf = 0;       // elements probed at the leaf (<= 16)
     int64_t t_per_nuc = 0;    // keys per nuclide
-    // bin bounds of every nuclide row (XS_SEARCH_H): [n_nuc][2^b_log2 + 1]
-    int32_t *bnd = nullptr;
+    // bin table of every nuclide row (XS_SEARCH_H): [n_nuc][2^b_log2]
+    struct BinEntry *bnd = nullptr;
     int32_t b_log2 = 0;
-    // bin bounds of the unionized energies (XS_SEARCH_H on XS_UNIONIZED): [2^u_log2 + 1]
-    int32_t *ubnd = nullptr;
+    // bin table of the unionized energies (XS_SEARCH_H on XS_UNIONIZED): [2^u_log2]
+    struct BinEntry *ubnd = nullptr;
     int32_t u_log2 = 0;
     double *U = nullptr;
     int32_t *IDX = nullptr;
@@ -114,13 +114,21 @@ struct DeviceGuard {
 };
 
 // ---- kernel arguments ----------------------------------------------------------------
+// One bin b of a sorted row A (XS_SEARCH_H): lo = L(b/2^k), cnt = L((b+1)/2^k) - lo,
+// e_next = A[lo + 1] -- for cnt <= 1 the lower index of any q in the bin is
+// lo + (cnt && e_next <= q) without touching the row.
+struct alignas(16) BinEntry {
+    int32_t lo;
+    int32_t cnt;
+    double e_next;
+};
 // Everything the lookup loop needs about nuclide j of material m, precomputed at grid
 // creation so the loop does one 32 B broadcast load instead of 64-bit row arithmetic.
 struct NucRef {
     const double *E;   // energy row of the nuclide            (E + nuc * n)
     const double *pts; // 48 B point records of the nuclide    (pts + nuc * n * 6)
     const double *T;   // separator tree of the nuclide, or NULL
-    const int32_t *B;  // bin bounds of the nuclide, or NULL
+    const BinEntry *B; // bin table of the nuclide, or NULL
     double conc;       // concs[m][j]
     int64_t nuc;       // nuclide id
 };
@@ -149,8 +157,8 @@ struct GridView {
     int32_t t_per_nuc;
     int32_t b_log2;   // XS_SEARCH_H bins = 2^b_log2 (0: no table)
     int32_t u_log2;   // unionized XS_SEARCH_H bins = 2^u_log2 (0: no table)
-    const int32_t *__restrict__ bnd;
-    const int32_t *__restrict__ ubnd;
+    const BinEntry *__restrict__ bnd;
+    const BinEntry *__restrict__ ubnd;
 };
 
 struct SampleView {
