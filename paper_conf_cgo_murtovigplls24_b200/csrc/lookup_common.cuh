@@ -259,6 +259,31 @@ __device__ __forceinline__ void accumulate_pair(const double *__restrict__ pts_r
     A.a4 = __fma_rn(__fma_rn(-f, __dsub_rn(h2.y, l2.y), h2.y), conc, A.a4);
 }
 
+// two pairs at once: all 12 loads issued before any arithmetic, the two divisions and
+// interpolations independent; accumulation in order a then b (reading R8)
+__device__ __forceinline__ void accumulate_pair2(const double *__restrict__ pa, int La, double ca,
+                                                 const double *__restrict__ pb, int Lb, double cb, double q, Acc &A)
+{
+    const double2 *p = reinterpret_cast<const double2 *>(pa) + (uint32_t)La * 3;
+    const double2 *s = reinterpret_cast<const double2 *>(pb) + (uint32_t)Lb * 3;
+    const double2 l0 = __ldg(p + 0), l1 = __ldg(p + 1), l2 = __ldg(p + 2);
+    const double2 h0 = __ldg(p + 3), h1 = __ldg(p + 4), h2 = __ldg(p + 5);
+    const double2 m0 = __ldg(s + 0), m1 = __ldg(s + 1), m2 = __ldg(s + 2);
+    const double2 k0 = __ldg(s + 3), k1 = __ldg(s + 4), k2 = __ldg(s + 5);
+    const double fa = __ddiv_rn(__dsub_rn(h0.x, q), __dsub_rn(h0.x, l0.x));
+    const double fb = __ddiv_rn(__dsub_rn(k0.x, q), __dsub_rn(k0.x, m0.x));
+    const double a0 = __fma_rn(-fa, __dsub_rn(h0.y, l0.y), h0.y), b0 = __fma_rn(-fb, __dsub_rn(k0.y, m0.y), k0.y);
+    const double a1 = __fma_rn(-fa, __dsub_rn(h1.x, l1.x), h1.x), b1 = __fma_rn(-fb, __dsub_rn(k1.x, m1.x), k1.x);
+    const double a2 = __fma_rn(-fa, __dsub_rn(h1.y, l1.y), h1.y), b2 = __fma_rn(-fb, __dsub_rn(k1.y, m1.y), k1.y);
+    const double a3 = __fma_rn(-fa, __dsub_rn(h2.x, l2.x), h2.x), b3 = __fma_rn(-fb, __dsub_rn(k2.x, m2.x), k2.x);
+    const double a4 = __fma_rn(-fa, __dsub_rn(h2.y, l2.y), h2.y), b4 = __fma_rn(-fb, __dsub_rn(k2.y, m2.y), k2.y);
+    A.a0 = __fma_rn(b0, cb, __fma_rn(a0, ca, A.a0));
+    A.a1 = __fma_rn(b1, cb, __fma_rn(a1, ca, A.a1));
+    A.a2 = __fma_rn(b2, cb, __fma_rn(a2, ca, A.a2));
+    A.a3 = __fma_rn(b3, cb, __fma_rn(a3, ca, A.a3));
+    A.a4 = __fma_rn(b4, cb, __fma_rn(a4, ca, A.a4));
+}
+
 // verification value (R10): 1 + first maximum, strict '>' from -1.0
 __device__ __forceinline__ uint32_t verify(const Acc &A)
 {

@@ -26,9 +26,13 @@ constexpr int kChunkIters = XS_CHUNK_ITERS; // 256-slot iterations per work chun
 #endif
 
 // OUTS: the call asked for macroscopic XS and/or indices; without it the bench/hash path
-// carries no output pointers (fewer live registers, no spills at 64 per thread)
-template <int GRID, int SEARCH, bool SORTED, bool OUTS>
-__global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W   ? XS_W_MIN_BLOCKS
+// carries no output pointers (fewer live registers, no spills at 64 per thread).
+// ILP2 (H on the nuclide grid only): two nuclides per iteration at 3 CTAs/SM -- chosen for
+// long nuclide lists (large tables: 1.06x), where it beats the extra occupancy of ILP1
+// (small tables: ILP1 is 1.05x faster).
+template <int GRID, int SEARCH, bool SORTED, bool OUTS, bool ILP2 = false>
+__global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
+                                             : SEARCH == XS_SEARCH_W ? XS_W_MIN_BLOCKS
                                              : SEARCH == XS_SEARCH_H ? XS_H_MIN_BLOCKS
                                                                      : 4)
     k_lookup(GridView gv, SampleView sv, SortedView so, Affine J_grid, double *__restrict__ out_,
@@ -41,6 +45,7 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W   ? XS_W_MIN_
 #define XS_PIPE_H 0
 #endif
     constexpr bool kPipeH = XS_PIPE_H && SEARCH == XS_SEARCH_H && GRID == XS_NUCLIDE;
+    constexpr bool kIlp2 = ILP2 && SEARCH == XS_SEARCH_H && GRID == XS_NUCLIDE;
     __shared__ uint32_t s_mb[kMaterials + 1];
     if constexpr (SORTED) {
         if (threadIdx.x <= kMaterials)
@@ -128,6 +133,32 @@ __global__ void __launch_bounds__(kFusedTpb, SEARCH == XS_SEARCH_W   ? XS_W_MIN_
                 if (out_idx)
                     out_idx[(size_t)r * gv.max_nucs + jn] = L;
                 accumulate_pair(rw.pts, L, q, rw.conc, A);
+            }
+        } else if (kIlp2 && active) {
+            // bin-bounded search, two nuclides per iteration: both rows, bins and 96 B
+            // gathers are independent, so their latency chains overlap; the accumulation
+            // stays in ascending nuclide order (reading R8), bit-identical to one at a time
+            const bool in01 = q >= 0.0 && q <= 1.0 && gv.b_log2 > 0;
+            const int bq = in01 ? bin_of(q, gv.b_log2) : 0;
+            const Bin full{0, gv.n - 2, 0.0};
+            int jn = 0;
+            for (; jn + 1 < nn; jn += 2) {
+                const Row ra = load_row(gv, row + jn), rb = load_row(gv, row + jn + 1);
+                const Bin ba = in01 ? load_bin(ra.B + bq) : full;
+                const Bin bb = in01 ? load_bin(rb.B + bq) : full;
+                const int La = bin_lower(ra.E, ba, q), Lb = bin_lower(rb.E, bb, q);
+                if (out_idx) {
+                    out_idx[(size_t)r * gv.max_nucs + jn] = La;
+                    out_idx[(size_t)r * gv.max_nucs + jn + 1] = Lb;
+                }
+                accumulate_pair2(ra.pts, La, ra.conc, rb.pts, Lb, rb.conc, q, A);
+            }
+            if (jn < nn) {
+                const Row ra = load_row(gv, row + jn);
+                const int La = bin_lower(ra.E, in01 ? load_bin(ra.B + bq) : full, q);
+                if (out_idx)
+                    out_idx[(size_t)r * gv.max_nucs + jn] = La;
+                accumulate_pair(ra.pts, La, q, ra.conc, A);
             }
         } else if (kPipeH && active) {
             // bin-bounded search, software-pipelined: the next nuclide's row and bin entry
@@ -217,6 +248,11 @@ void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, c
     FusedFn f = grid_type == XS_NUCLIDE     ? pick_g<XS_NUCLIDE>(search, sorted, outs)
                 : grid_type == XS_UNIONIZED ? pick_g<XS_UNIONIZED>(search, sorted, outs)
                                             : pick_g<XS_HASH>(search, sorted, outs);
+    if (grid_type == XS_NUCLIDE && search == XS_SEARCH_H && sorted && gv.max_nucs > 64) {
+        f = outs ? k_lookup<XS_NUCLIDE, XS_SEARCH_H, true, true, true>
+                 : k_lookup<XS_NUCLIDE, XS_SEARCH_H, true, false, true>;
+        blocks = std::min(blocks, blocks / 4 * 3 > 0 ? blocks / 4 * 3 : blocks); // one wave at 3 CTAs/SM
+    }
     f<<<blocks, tpb, 0, stream>>>(gv, sv, so, J_grid, out, out_idx, stats);
     XS_CUDA_TRY(cudaGetLastError());
 }

@@ -1,0 +1,44 @@
+"""compute-sanitizer over the tiny configuration: memcheck, racecheck,
+initcheck and synccheck on every kernel of grid creation, sorting and lookup."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SAN = "/usr/local/cuda/bin/compute-sanitizer"
+
+SCRIPT = r"""
+import sys; sys.path.insert(0, %r)
+import torch
+import paper_conf_cgo_murtovigplls24_b200 as xs
+for gt in (0, 1, 2):
+    g = xs.Grid(68, 200, gt, 42)
+    for search in ("M", "U2", "W", "H"):
+        for sort in ("none", "material_energy"):
+            out, st = g.macro_xs(0, 3000, 1070, search=search, sort=sort)
+    g.indices(5, 1000, 1070, sort="material_energy", split=True)
+    g.sample(0, 100, 1070)
+    g.search_points([0.5, 1.0, -1.0], [0, 1, 2], "H")
+    g.checksum()
+    g.close()
+print("SANITIZED")
+""" % ROOT
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "initcheck", "synccheck"])
+def test_compute_sanitizer(tool):
+    if not os.path.exists(SAN):
+        pytest.skip("compute-sanitizer not installed")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    args = [SAN, "--tool", tool, "--error-exitcode", "9"]
+    if tool == "memcheck":
+        args += ["--leak-check", "no"]
+    r = subprocess.run(args + [sys.executable, "-c", SCRIPT], capture_output=True, text=True, timeout=1800)
+    assert r.returncode == 0 and "SANITIZED" in r.stdout, (r.stdout[-3000:], r.stderr[-3000:])
+    text = r.stdout + r.stderr
+    assert "ERROR SUMMARY: 0 errors" in text or "(0 errors, 0 warnings)" in text, text[-2000:]
