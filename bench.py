@@ -257,6 +257,13 @@ def run_ours(a, w):
                  "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
     if a.ab:
         for _ in range(2):
+            step(search="H", sort="history")
+        ms, sts = timed_steps(a.ab_steps, search="H", sort="history")
+        ms_max = driver.max_over_ranks(sum(ms))
+        ab["H/history (XSBench history order, 34 lookups/particle)"] = {
+            "value": R.world * count * a.ab_steps / (ms_max / 1e3),
+            "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
+        for _ in range(2):
             step(search="M", sort="none")
         ms, sts = timed_steps(a.ab_steps, search="M", sort="none")
         ms_max = driver.max_over_ranks(sum(ms))

@@ -79,7 +79,11 @@ enum {
 enum {
     XS_SORT_NONE = 0,            /* one thread per lookup in index order (XSBench baseline)  */
     XS_SORT_MATERIAL = 1,        /* bucket by material                                       */
-    XS_SORT_MATERIAL_ENERGY = 2  /* bucket by (material, energy bucket): coherent warps       */
+    XS_SORT_MATERIAL_ENERGY = 2, /* bucket by (material, energy bucket): coherent warps      */
+    XS_SORT_HISTORY = 3          /* XSBench history order: one thread
+                                    per particle running opts.history_len consecutive lookups,
+                                    its stream continuing from one lookup to the next (lookup
+                                    i of the range = particle i / len, step i % len)        */
 };
 
 /* Flags. */
@@ -99,7 +103,7 @@ typedef struct xs_opts {
                             energy_bins buckets are shared out in proportion to each
                             material's expected (lookup, nuclide) pairs                 */
     uint32_t flags;      /* XS_FLAG_*                                                   */
-    int32_t reserved;
+    int32_t history_len; /* XS_SORT_HISTORY: lookups per particle; 0 = default (34)     */
 } xs_opts;
 
 typedef struct xs_stats {

@@ -72,7 +72,7 @@ void xs_opts_default(xs_opts *o)
     o->block = 0;
     o->energy_bins = 0;
     o->flags = 0;
-    o->reserved = 0;
+    o->history_len = 0;
 }
 
 const char *xs_last_error(void) { return t_err.c_str(); }

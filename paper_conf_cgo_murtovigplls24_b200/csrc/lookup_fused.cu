@@ -214,6 +214,81 @@ __global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
     reduce_stats<kFusedTpb>(my_hash, my_pairs, stats);
 }
 
+// XSBench history order: thread p runs particle p's `hl` lookups one after the other, its
+// stream continuing (two draws per lookup: the 2-step affine map); lookup i of the range
+// is particle i / hl, step i % hl, so results equal the event order's exactly
+template <int GRID, int SEARCH, bool OUTS>
+__global__ void __launch_bounds__(kFusedTpb, 4)
+    k_history(GridView gv, SampleView sv, int hl, Affine J2, double *__restrict__ out_, int32_t *__restrict__ out_idx_,
+              unsigned long long *__restrict__ stats)
+{
+    double *__restrict__ out = OUTS ? out_ : nullptr;
+    int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
+    uint32_t my_hash = 0, my_pairs = 0;
+    const int64_t count = sv.count;
+    const int64_t particles = (count + hl - 1) / hl;
+    for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < particles;
+         p += (int64_t)gridDim.x * blockDim.x) {
+        uint64_t s = lookup_state(sv, p * hl); // Listing-7 jump once per particle
+        const int64_t i_end = min(count, (p + 1) * hl);
+        for (int64_t i = p * hl; i < i_end; i++) {
+            double q;
+            int mat;
+            sample_lookup(s, sv, q, mat);
+            s = lcg_apply(J2, s);
+            const int nn = __ldg(gv.num_nucs + mat);
+            const int row = mat * gv.max_nucs;
+            const int e_union = union_index<GRID, SEARCH>(gv, q);
+            Acc A;
+            for (int jn = 0; jn < nn; jn++) {
+                const Row rw = load_row(gv, row + jn);
+                const int L = lower_index<GRID, SEARCH>(gv, rw, q, e_union);
+                if (out_idx)
+                    out_idx[(size_t)i * gv.max_nucs + jn] = L;
+                accumulate_pair(rw.pts, L, q, rw.conc, A);
+            }
+            my_hash += verify(A);
+            my_pairs += (uint32_t)nn;
+            if (out)
+                store_macro(out, (uint32_t)i, A);
+        }
+    }
+    reduce_stats<kFusedTpb>(my_hash, my_pairs, stats);
+}
+
+using HistFn = void (*)(GridView, SampleView, int, Affine, double *, int32_t *, unsigned long long *);
+
+template <int GRID> static HistFn pick_hist_g(int search, bool outs)
+{
+#define XS_HIST_CASE(S)                                                                                      \
+    case S: return outs ? k_history<GRID, S, true> : k_history<GRID, S, false>;
+    switch (search) {
+        XS_HIST_CASE(XS_SEARCH_M)
+        XS_HIST_CASE(XS_SEARCH_U1)
+        XS_HIST_CASE(XS_SEARCH_U2)
+        XS_HIST_CASE(XS_SEARCH_U4)
+        XS_HIST_CASE(XS_SEARCH_U8)
+        XS_HIST_CASE(XS_SEARCH_B)
+        XS_HIST_CASE(XS_SEARCH_M2)
+        XS_HIST_CASE(XS_SEARCH_M4)
+        XS_HIST_CASE(XS_SEARCH_M8)
+        XS_HIST_CASE(XS_SEARCH_W)
+    default: return outs ? k_history<GRID, XS_SEARCH_H, true> : k_history<GRID, XS_SEARCH_H, false>;
+    }
+#undef XS_HIST_CASE
+}
+
+void launch_history(int grid_type, int search, int hl, int blocks, cudaStream_t stream, const GridView &gv,
+                    const SampleView &sv, double *out, int32_t *out_idx, unsigned long long *stats)
+{
+    const bool outs = out || out_idx;
+    HistFn f = grid_type == XS_NUCLIDE     ? pick_hist_g<XS_NUCLIDE>(search, outs)
+               : grid_type == XS_UNIONIZED ? pick_hist_g<XS_UNIONIZED>(search, outs)
+                                           : pick_hist_g<XS_HASH>(search, outs);
+    f<<<blocks, kFusedTpb, 0, stream>>>(gv, sv, hl, lcg_jump(2), out, out_idx, stats);
+    XS_CUDA_TRY(cudaGetLastError());
+}
+
 using FusedFn = void (*)(GridView, SampleView, SortedView, Affine, double *, int32_t *, unsigned long long *);
 
 template <int GRID, int SEARCH> static FusedFn pick_s(bool sorted, bool outs)

@@ -110,7 +110,10 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
                  int32_t *out_idx, xs_stats *st)
 {
     XS_CHECK_ARG(o.search >= 0 && o.search < XS_SEARCH_COUNT, "opts.search out of range");
-    XS_CHECK_ARG(o.sort >= XS_SORT_NONE && o.sort <= XS_SORT_MATERIAL_ENERGY, "opts.sort out of range");
+    XS_CHECK_ARG(o.sort >= XS_SORT_NONE && o.sort <= XS_SORT_HISTORY, "opts.sort out of range");
+    const bool history = o.sort == XS_SORT_HISTORY;
+    const int hl = o.history_len ? o.history_len : 34;
+    XS_CHECK_ARG(!history || (hl >= 1 && hl <= (1 << 20)), "opts.history_len must be in [1, 2^20]");
     const int tpb = o.block ? o.block : 256;
     XS_CHECK_ARG(tpb == 64 || tpb == 128 || tpb == 256, "opts.block must be 64, 128 or 256");
     const int nb = (o.sort == XS_SORT_MATERIAL_ENERGY) ? (o.energy_bins ? o.energy_bins : kMaxEnergyBins) : 1;
@@ -118,7 +121,7 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
     XS_CHECK_ARG(nb_log2 >= 0 && nb <= kMaxEnergyBins, "opts.energy_bins must be a power of two <= 4096");
     cudaStream_t stream = (cudaStream_t)o.stream;
     const bool timing = (o.flags & XS_FLAG_TIMING) != 0;
-    const bool sorted = o.sort != XS_SORT_NONE;
+    const bool sorted = o.sort == XS_SORT_MATERIAL || o.sort == XS_SORT_MATERIAL_ENERGY;
     const bool fused = !sorted || !(o.flags & XS_FLAG_SPLIT);
     const bool host_out = out_macro && !is_device_accessible(out_macro);
     int64_t chunk = fused ? (sorted ? kChunkSorted : kChunkFused) : kChunkSplit;
@@ -128,6 +131,8 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         const int64_t nch = (count + chunk - 1) / chunk;
         chunk = (count + nch - 1) / nch;
     }
+    if (history && count > chunk) // whole particles per chunk: history stream positions stay global
+        chunk = std::max<int64_t>(hl, chunk / hl * hl);
     const GridView gv = make_view(g);
     int launches = 0;
     double sample_ms = 0, lookup_ms = 0, search_ms = 0, copy_ms = 0;
@@ -183,7 +188,14 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         }
         XS_CUDA_TRY(cudaEventRecord(g.ev[2], stream));
         XS_CUDA_TRY(cudaEventRecord(g.ev[3], stream));
-        if (fused) {
+        if (history) {
+            // chunk boundaries are multiples of hl (chunk >= 2^22 > hl, rounded below), so a
+            // particle never straddles two chunks
+            const int64_t particles = (cn + hl - 1) / hl;
+            launch_history(g.grid_type, o.search, hl, blocks_for(particles, 256, 32), stream, gv, sv, outp, idxp,
+                           stats);
+            launches += 1;
+        } else if (fused) {
             // sorted: a persistent grid (one resident wave) pulling work chunks;
             // unsorted: 4 waves of grid-stride CTAs
             const int blocks = blocks_for(cn, tpb, sorted ? (1024 / tpb) : (2048 / tpb) * 4);

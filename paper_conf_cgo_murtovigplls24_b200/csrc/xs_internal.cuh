@@ -205,6 +205,10 @@ void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, c
                   const GridView &gv, const SampleView &sv, const SortedView &so, Affine J_grid, double *out,
                   int32_t *out_idx, unsigned long long *stats);
 
+// lookup_fused.cu: XSBench history order (XS_SORT_HISTORY)
+void launch_history(int grid_type, int search, int hl, int blocks, cudaStream_t stream, const GridView &gv,
+                    const SampleView &sv, double *out, int32_t *out_idx, unsigned long long *stats);
+
 // lookup_split.cu: k_search (every pair's lower index into the pair buffer; the paper's
 // loop, alone, at full occupancy) then k_interp (gather + interpolate + accumulate)
 void launch_search(int grid_type, int search, int blocks, cudaStream_t stream, const GridView &gv,

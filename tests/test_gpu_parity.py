@@ -88,7 +88,7 @@ def test_sample_bitexact(tiny, first):
 # ------------------------------------------------------------------ tiny: full cross product
 # (sort, split): the XSBench order; sorted + the fused kernel; sorted + k_search/k_interp
 PIPES = [("none", False), ("material", False), ("material_energy", False), ("material", True),
-         ("material_energy", True)]
+         ("material_energy", True), ("history", False)]
 
 
 @pytest.mark.parametrize("gt", [0, 1, 2])
@@ -130,6 +130,18 @@ def test_energy_bins_and_block(tiny, bins, block):
     out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, sort="material_energy", energy_bins=bins, block=block)
     assert st.hash == ref["hash"]
     assert np.array_equal(out.cpu().numpy(), ref["macro"])
+
+
+@pytest.mark.parametrize("hl", [1, 7, 34, 1000, 200_000])
+def test_history_order_equals_event_order(tiny, hl):
+    """XSBench history order (one particle = hl consecutive lookups, continuing stream):
+    lookup i is particle i // hl, step i % hl, so every output equals the event order's."""
+    g, P, ref = tiny[1]
+    for first, count in [(0, 100_000), (13, 99_987)]:
+        out, st = g.macro_xs(first, count, LOOKUP_SEED, sort="history", history_len=hl)
+        r = ref if first == 0 else P.run_range(LOOKUP_SEED, first, count)
+        assert st.hash == r["hash"] and st.pairs == r["pairs"]
+        assert np.array_equal(out.cpu().numpy(), r["macro"])
 
 
 def test_host_outputs(tiny, xs):
@@ -217,6 +229,8 @@ def test_small_full_hash(xs, oracle_mod):
             st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search=search, split=split)
             assert st.hash == ref["hash"] and st.pairs == ref["pairs"]
     st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search="U2", sort="none")
+    assert st.hash == ref["hash"]
+    st = g.lookup_range(0, w.lookups, LOOKUP_SEED, sort="history", history_len=34)
     assert st.hash == ref["hash"]
     _sampled_check(g, P, w.lookups)
 
