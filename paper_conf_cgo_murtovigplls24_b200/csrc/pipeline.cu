@@ -7,6 +7,7 @@
 // fused path reads the material bases from device memory (no host round trip); the split
 // path brings them back (52 B) to size the pair buffer exactly.
 #include <algorithm>
+#include <cstdlib>
 
 #include "lookup_common.cuh"
 
@@ -127,6 +128,13 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
     int64_t chunk = fused ? (sorted ? kChunkSorted : kChunkFused) : kChunkSplit;
     if (host_out)
         chunk = std::min(chunk, kChunkHost);
+    // test hook: XS_TEST_MAX_CHUNK forces small chunks so the chunk-boundary paths (offsets,
+    // host-output double buffering, history alignment) are checked at tiny sizes
+    if (const char *env = std::getenv("XS_TEST_MAX_CHUNK")) {
+        const long long v = std::atoll(env);
+        if (v > 0)
+            chunk = std::min<int64_t>(chunk, v);
+    }
     if (count > chunk) { // equal chunks (no small tail chunk)
         const int64_t nch = (count + chunk - 1) / chunk;
         chunk = (count + nch - 1) / nch;
