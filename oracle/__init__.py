@@ -19,6 +19,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "xs_oracle.c")
+_SRCS = [_SRC, os.path.join(_HERE, "bezier_oracle.c")]
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lock = threading.Lock()
 _lib = None
@@ -29,9 +30,9 @@ HASH_BINS = 10000
 
 def build(force: bool = False) -> str:
     """Compile oracle/liboracle.so (plain C, no CUDA)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS):
         cmd = ["gcc", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared",
-               "-std=c99", "-Wall", "-o", _LIB + ".tmp", _SRC, "-lm"]
+               "-std=c99", "-Wall", "-o", _LIB + ".tmp", *_SRCS, "-lm"]
         subprocess.run(cmd, check=True)
         os.replace(_LIB + ".tmp", _LIB)
     return _LIB
@@ -80,6 +81,14 @@ def lib():
                 "or_run_range": (C.c_int, [vp, u64, i64, i64, vp, vp, vp, vp, vp, vp, i32]),
                 "or_run_indices": (C.c_int, [vp, u64, vp, i64, vp, vp, i32]),
                 "or_max_threads": (i32, []),
+                "ob_blend_loop_f64": (dbl, [C.c_int, C.c_int]),
+                "ob_blend_loop_f32": (C.c_float, [C.c_int, C.c_int]),
+                "ob_bezier_blend_f64": (dbl, [C.c_int, dbl, C.c_int]),
+                "ob_bezier_blend_f32": (C.c_float, [C.c_int, C.c_float, C.c_int]),
+                "ob_surface_f64": (None, [C.c_int, C.c_int, i64, i64, vp, vp]),
+                "ob_surface_f32": (None, [C.c_int, C.c_int, i64, i64, vp, vp]),
+                "ob_surface_points_f64": (None, [C.c_int, C.c_int, i64, i64, vp, i64, vp, vp, vp]),
+                "ob_surface_points_f32": (None, [C.c_int, C.c_int, i64, i64, vp, i64, vp, vp, vp]),
             }
             for name, (res, args) in sig.items():
                 f = getattr(L, name)
@@ -258,3 +267,38 @@ class Problem:
 
 def max_threads() -> int:
     return lib().or_max_threads()
+
+
+# ---------------------------------------------------------------- bezier-surface (Listing 2)
+def blend_loop(k: int, n: int, dtype=np.float64) -> float:
+    """Listing 2 from blend = 1 (reading BZ1)."""
+    f = lib().ob_blend_loop_f64 if np.dtype(dtype) == np.float64 else lib().ob_blend_loop_f32
+    return f(k, n)
+
+
+def bezier_blend(k: int, mu: float, n: int, dtype=np.float64) -> float:
+    """Listing 2 times mu^k (1-mu)^(n-k) (reading BZ2)."""
+    f = lib().ob_bezier_blend_f64 if np.dtype(dtype) == np.float64 else lib().ob_bezier_blend_f32
+    return f(k, mu, n)
+
+
+def bezier_surface(P: np.ndarray, res_i: int, res_j: int) -> np.ndarray:
+    """The surface (readings BZ3-BZ5) over the control net P[(ni+1), (nj+1), 3] in P's dtype."""
+    P = np.ascontiguousarray(P)
+    ni, nj = P.shape[0] - 1, P.shape[1] - 1
+    out = np.zeros((res_i, res_j, 3), P.dtype)
+    f = lib().ob_surface_f64 if P.dtype == np.float64 else lib().ob_surface_f32
+    f(ni, nj, res_i, res_j, _p(P), _p(out))
+    return out
+
+
+def bezier_surface_points(P: np.ndarray, res_i: int, res_j: int, ii, jj) -> np.ndarray:
+    """surface(ii[t], jj[t]) for sampled points of a res_i x res_j surface."""
+    P = np.ascontiguousarray(P)
+    ii = np.ascontiguousarray(ii, np.int64)
+    jj = np.ascontiguousarray(jj, np.int64)
+    ni, nj = P.shape[0] - 1, P.shape[1] - 1
+    out = np.zeros((len(ii), 3), P.dtype)
+    f = lib().ob_surface_points_f64 if P.dtype == np.float64 else lib().ob_surface_points_f32
+    f(ni, nj, res_i, res_j, _p(P), len(ii), _p(ii), _p(jj), _p(out))
+    return out

@@ -44,3 +44,37 @@ WORKLOADS = {
 # Mean nuclides per lookup under pick_mat's effective distribution (SURVEY.md §8
 # notation; [derived]); used only to state algorithmic bytes, never in results.
 MEAN_NUCS = {68: 15.490, 355: 55.383}
+
+
+# ---------------------------------------------------------------- bezier-surface (NEXT 4)
+# The second u&u loop of the paper (Listing 2), run as a synthetic A/B.
+# Table I runs bezier-surface with "-n 4096"; reading BZ3 takes
+# that as a 4096 x 4096 output surface over a (NI+1) x (NJ+1) control net.
+@dataclass(frozen=True)
+class BezierWorkload:
+    name: str
+    ni: int
+    nj: int
+    res_i: int
+    res_j: int
+    note: str
+
+
+BEZIER_SEED = 7
+BEZIER_WORKLOADS = {
+    "tiny": BezierWorkload("tiny", 5, 4, 61, 37, "oracle-sized, ragged against the 16 x 16 tiles"),
+    "paper": BezierWorkload("paper", 5, 4, 4096, 4096, "-n 4096, NI=5, NJ=4 (reading BZ3)"),
+    "deep": BezierWorkload("deep", 16, 16, 2048, 2048, "17 x 17 net: 16-trip Listing-2 loops"),
+}
+
+
+def bezier_control_net(ni: int, nj: int, seed: int = BEZIER_SEED, dtype="float64"):
+    """Seeded control net P[(ni+1), (nj+1), 3]: a jittered lattice (x = ki, y = kj) with
+    uniform heights in [0, 1) -- the shape of a terrain/patch input.  Input data only."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    P = np.zeros((ni + 1, nj + 1, 3), np.float64)
+    P[..., 0] = np.arange(ni + 1)[:, None] + rng.uniform(-0.25, 0.25, (ni + 1, nj + 1))
+    P[..., 1] = np.arange(nj + 1)[None, :] + rng.uniform(-0.25, 0.25, (ni + 1, nj + 1))
+    P[..., 2] = rng.random((ni + 1, nj + 1))
+    return P.astype(dtype)
