@@ -1,0 +1,36 @@
+"""Summarise an `ncu --metrics gpu__time_duration.sum --csv --log-file X.csv` launch list
+into a markdown table (kernel, launches, mean duration, share of the lookup step).
+usage: python tools/launch_summary.py LAUNCHES.csv TITLE > profiles/<round>_launches_<w>.md
+Step kernels are the sort kernels and k_lookup; everything else is setup or L2 flush."""
+import csv
+import sys
+from collections import OrderedDict
+
+STEP = ("k_bucket_count", "k_bucket_colscan", "k_bucket_base", "k_bucket_scatter", "k_bucket_gather",
+        "k_lookup", "k_history", "k_search", "k_interp")
+UNIT = {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3}
+
+
+def main():
+    path, title = sys.argv[1], sys.argv[2]
+    lines = [l for l in open(path) if l.startswith('"')]
+    rows = list(csv.DictReader(lines))
+    agg = OrderedDict()
+    for r in rows:
+        if r.get("Metric Name") != "gpu__time_duration.sum":
+            continue
+        us = float(r["Metric Value"].replace(",", "")) * UNIT.get(r["Metric Unit"], 1e-3)
+        a = agg.setdefault(r["Kernel Name"][:90], [0, 0.0])
+        a[0] += 1
+        a[1] += us
+    step_total = sum(v[1] for k, v in agg.items() if any(s in k for s in STEP))
+    print(f"# {title}\n")
+    print("`ncu --metrics gpu__time_duration.sum --clock-control none` (serialised, cold: compare SHARES)\n")
+    print("| kernel | launches | mean us (ncu) | share of a step |\n|---|---|---|---|")
+    for k, (n, us) in agg.items():
+        share = f"{100 * us / step_total:.1f}%" if any(s in k for s in STEP) and step_total else "setup / L2 flush / e2e"
+        print(f"| `{k}` | {n} | {us / n:.1f} | {share} |")
+
+
+if __name__ == "__main__":
+    main()
