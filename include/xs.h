@@ -203,6 +203,45 @@ int xs_grid_export(const xs_grid *grid, double *E, double *X, int32_t *mats, dou
  * H [hash_bins][n_nuclides] (XS_HASH); host arrays, each may be NULL. */
 int xs_grid_export_aux(const xs_grid *grid, double *U, int32_t *IDX, int32_t *H);
 
+/* ---------------------------------------------------------------------------------
+ * The paper's second u&u example: the bezier-surface loop (Listing 2, PAPER.md:160-185;
+ * SURVEY.md §8f NEXT 4; DESIGN.md §6.9 and readings BZ1-BZ5).  Off the north star: a
+ * synthetic A/B of the loop transformation.  BezierBlend(k, mu, n) = Listing 2 (from
+ * blend = 1, nn = n, kn = k, nkn = n - k) * mu^k * (1 - mu)^(n - k), powers by repeated
+ * multiplication; surface(i, j)[c] = sum_ki sum_kj (P[ki][kj][c] * B(ki, mu_i, ni)) *
+ * B(kj, mu_j, nj), ki-major, mu_i = i / (res_i - 1).  Every variant performs the same
+ * floating-point operations in the same order: results are bit-identical across variants
+ * and to the CPU oracle.
+ * --------------------------------------------------------------------------------- */
+enum {
+    XS_BZ_M = 0,  /* Listing 2 as written                                              */
+    XS_BZ_M2 = 1, /* unroll-only x2                                                    */
+    XS_BZ_U1 = 2, /* unmerge-only                                                      */
+    XS_BZ_U2 = 3, /* u&u x2: the unrolled copy specialised per path (Figure 5)         */
+    XS_BZ_S = 4,  /* one loop per condition state (the u -> infinity limit)            */
+    XS_BZ_T = 5,  /* B200 design: per-tile blends in shared memory, then contraction   */
+    XS_BZ_COUNT = 6
+};
+enum { XS_F64 = 0, XS_F32 = 1 }; /* element type of the bezier buffers */
+
+/* Evaluate a res_i x res_j bezier surface.
+ *   ni, nj   in [0, 32]: the control net has (ni+1) x (nj+1) points
+ *   res_i, res_j >= 2, res_i * res_j < 2^40
+ *   ctrl     device, [(ni+1)][(nj+1)][3] of dtype (row-major)
+ *   out      device, [res_i][res_j][3] of dtype (written in full)
+ *   dtype    XS_F64 or XS_F32 (every operation rounded in that type, no contraction)
+ *   variant  XS_BZ_*
+ * Enqueued on `stream` and synchronised before returning.  XS_EINVAL on a bad argument. */
+int xs_bezier_surface(int32_t ni, int32_t nj, int64_t res_i, int64_t res_j, int32_t dtype, int32_t variant,
+                      const void *ctrl, void *out, void *stream);
+
+/* Loop-level parity: out[t] = BezierBlend(k[t], mu[t], n[t]), or the bare Listing-2
+ * loop value when mu is NULL.  k, n, mu, out: device arrays of length count (mu and out
+ * of dtype).  The loop runs n[t] trips: callers keep 0 <= k[t] and n[t] <= 2^20
+ * (device contents are not inspected).  XS_BZ_T evaluates the loop as XS_BZ_M. */
+int xs_bezier_blend(int64_t count, const int32_t *k, const int32_t *n, const void *mu, int32_t dtype,
+                    int32_t variant, void *out, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

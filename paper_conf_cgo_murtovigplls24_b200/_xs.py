@@ -35,6 +35,10 @@ XS_FLAG_SPLIT = 2
 
 SEARCH_NAMES = {"M": 0, "U1": 1, "U2": 2, "U4": 3, "U8": 4, "B": 5, "M2": 6, "M4": 7, "M8": 8, "W": 9, "H": 10}
 SORT_NAMES = {"none": 0, "material": 1, "material_energy": 2, "history": 3}
+XS_BZ_M, XS_BZ_M2, XS_BZ_U1, XS_BZ_U2, XS_BZ_S, XS_BZ_T = range(6)
+XS_BZ_COUNT = 6
+XS_F64, XS_F32 = 0, 1
+BZ_NAMES = {"M": 0, "M2": 1, "U1": 2, "U2": 3, "S": 4, "T": 5}
 
 
 class xs_opts(C.Structure):
@@ -73,6 +77,8 @@ _SIGS = {
     "xs_grid_get_info": (C.c_int, [_vp, C.POINTER(xs_grid_info)]),
     "xs_grid_export": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
     "xs_grid_export_aux": (C.c_int, [_vp, _vp, _vp, _vp]),
+    "xs_bezier_surface": (C.c_int, [_i32, _i32, _i64, _i64, _i32, _i32, _vp, _vp, _vp]),
+    "xs_bezier_blend": (C.c_int, [_i64, _vp, _vp, _vp, _i32, _i32, _vp, _vp]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -177,3 +183,12 @@ def xs_grid_export(grid: int, E=None, X=None, mats=None, concs=None) -> None:
 
 def xs_grid_export_aux(grid: int, U=None, IDX=None, H=None) -> None:
     _check(_lib.xs_grid_export_aux(grid, _ptr(U), _ptr(IDX), _ptr(H)))
+
+
+def xs_bezier_surface(ni: int, nj: int, res_i: int, res_j: int, dtype: int, variant: int, ctrl, out,
+                      stream: int | None = None) -> None:
+    _check(_lib.xs_bezier_surface(ni, nj, res_i, res_j, dtype, variant, _ptr(ctrl), _ptr(out), stream))
+
+
+def xs_bezier_blend(count: int, k, n, mu, dtype: int, variant: int, out, stream: int | None = None) -> None:
+    _check(_lib.xs_bezier_blend(count, _ptr(k), _ptr(n), _ptr(mu), dtype, variant, _ptr(out), stream))

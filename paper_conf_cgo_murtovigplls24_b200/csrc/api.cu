@@ -268,4 +268,34 @@ int xs_grid_export_aux(const xs_grid *grid, double *U, int32_t *IDX, int32_t *H)
     });
 }
 
+int xs_bezier_surface(int32_t ni, int32_t nj, int64_t res_i, int64_t res_j, int32_t dtype, int32_t variant,
+                      const void *ctrl, void *out, void *stream)
+{
+    return guarded([&] {
+        XS_CHECK_ARG(ni >= 0 && ni <= 32 && nj >= 0 && nj <= 32, "ni and nj must be in [0, 32]");
+        XS_CHECK_ARG(res_i >= 2 && res_j >= 2, "res_i and res_j must be >= 2");
+        XS_CHECK_ARG(res_i < (int64_t(1) << 40) / res_j, "res_i * res_j must be < 2^40");
+        XS_CHECK_ARG(dtype == XS_F64 || dtype == XS_F32, "dtype must be XS_F64 or XS_F32");
+        XS_CHECK_ARG(variant >= 0 && variant < XS_BZ_COUNT, "unknown bezier variant");
+        XS_CHECK_ARG(ctrl != nullptr && out != nullptr, "ctrl and out are required");
+        const cudaStream_t s = (cudaStream_t)stream;
+        run_bezier_surface(ni, nj, res_i, res_j, dtype, variant, ctrl, out, s);
+        XS_CUDA_TRY(cudaStreamSynchronize(s));
+    });
+}
+
+int xs_bezier_blend(int64_t count, const int32_t *k, const int32_t *n, const void *mu, int32_t dtype,
+                    int32_t variant, void *out, void *stream)
+{
+    return guarded([&] {
+        XS_CHECK_ARG(count >= 0, "count must be >= 0");
+        XS_CHECK_ARG((k && n && out) || count == 0, "k, n and out are required");
+        XS_CHECK_ARG(dtype == XS_F64 || dtype == XS_F32, "dtype must be XS_F64 or XS_F32");
+        XS_CHECK_ARG(variant >= 0 && variant < XS_BZ_COUNT, "unknown bezier variant");
+        const cudaStream_t s = (cudaStream_t)stream;
+        run_bezier_blend(count, k, n, mu, dtype, variant, out, s);
+        XS_CUDA_TRY(cudaStreamSynchronize(s));
+    });
+}
+
 } // extern "C"

@@ -18,6 +18,14 @@ constexpr int kFusedTpb = 256;
 #define XS_CHUNK_ITERS 4
 #endif
 constexpr int kChunkIters = XS_CHUNK_ITERS; // 256-slot iterations per work chunk (sorted)
+#ifndef XS_WARP_QUEUE
+#define XS_WARP_QUEUE 0
+#endif
+#ifndef XS_WARP_ITERS
+#define XS_WARP_ITERS 8
+#endif
+constexpr bool kWarpQueue = XS_WARP_QUEUE; // each warp pulls its own chunks (no CTA barrier)
+constexpr int kWarpIters = XS_WARP_ITERS;  // 32-slot iterations per warp chunk
 #ifndef XS_W_MIN_BLOCKS
 #define XS_W_MIN_BLOCKS 4
 #endif
@@ -61,15 +69,24 @@ __global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
     // narrow band (L2 reuse when the grid does not fit), and the load balances itself.
     // Unsorted: grid-stride over the chunk (XSBench order).
     __shared__ int s_chunk;
-    const int csize = SORTED ? kChunkIters * (int)blockDim.x : 0;
+    const int csize = !SORTED ? 0 : kWarpQueue ? kWarpIters * 32 : kChunkIters * (int)blockDim.x;
+    const int tpos = kWarpQueue ? lane : (int)threadIdx.x; // position inside a chunk
     int j0, jend, G;
     if constexpr (SORTED) {
-        if (threadIdx.x == 0)
-            s_chunk = atomicAdd(so.work, 1);
-        __syncthreads();
-        j0 = s_chunk * csize + threadIdx.x;
-        jend = min(count, s_chunk * csize + csize);
-        G = blockDim.x;
+        int c;
+        if constexpr (kWarpQueue) {
+            if (lane == 0)
+                c = atomicAdd(so.work, 1);
+            c = __shfl_sync(0xffffffffu, c, 0);
+        } else {
+            if (threadIdx.x == 0)
+                s_chunk = atomicAdd(so.work, 1);
+            __syncthreads();
+            c = s_chunk;
+        }
+        j0 = c * csize + tpos;
+        jend = min(count, c * csize + csize);
+        G = kWarpQueue ? 32 : blockDim.x;
     } else {
         j0 = blockIdx.x * blockDim.x + threadIdx.x;
         jend = count;
@@ -85,7 +102,7 @@ __global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
     }
     for (;;) {
         if constexpr (SORTED) {
-            if (j0 - (int)threadIdx.x >= count)
+            if (j0 - tpos >= count)
                 break;
             if (j0 < jend) {
                 r_next = ld_stream(so.slot + j0, pol);
@@ -203,12 +220,20 @@ __global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
         if constexpr (!SORTED)
             break;
         else { // next chunk
-            __syncthreads();
-            if (threadIdx.x == 0)
-                s_chunk = atomicAdd(so.work, 1);
-            __syncthreads();
-            j0 = s_chunk * csize + threadIdx.x;
-            jend = min(count, s_chunk * csize + csize);
+            int c;
+            if constexpr (kWarpQueue) {
+                if (lane == 0)
+                    c = atomicAdd(so.work, 1);
+                c = __shfl_sync(0xffffffffu, c, 0);
+            } else {
+                __syncthreads();
+                if (threadIdx.x == 0)
+                    s_chunk = atomicAdd(so.work, 1);
+                __syncthreads();
+                c = s_chunk;
+            }
+            j0 = c * csize + tpos;
+            jend = min(count, c * csize + csize);
         }
     }
     reduce_stats<kFusedTpb>(my_hash, my_pairs, stats);

@@ -221,6 +221,10 @@ constexpr int kInterpTpb = 256;
 // pipeline.cu
 void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
                  int32_t *out_idx, xs_stats *st);
+void run_bezier_surface(int ni, int nj, int64_t res_i, int64_t res_j, int dtype, int variant, const void *P,
+                        void *out, cudaStream_t s);
+void run_bezier_blend(int64_t count, const int32_t *k, const int32_t *n, const void *mu, int dtype, int variant,
+                      void *out, cudaStream_t s);
 void run_sample(Grid &g, int64_t first, int64_t count, uint64_t seed, double *q, int32_t *mat, cudaStream_t s);
 void run_search_points(Grid &g, int64_t count, const double *q, const int32_t *nuc, int search, int32_t *out,
                        cudaStream_t s);
