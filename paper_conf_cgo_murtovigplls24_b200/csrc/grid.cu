@@ -82,6 +82,23 @@ __global__ void k_fill_points(uint64_t seed, int64_t N, int32_t n, double *__res
     }
 }
 
+// interval records (XS_IV): iv[i] for interval L = i mod (n-1) of nuclide i / (n-1)
+__global__ void k_iv_build(int64_t NI, int32_t n, const double *__restrict__ pts, double *__restrict__ iv)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < NI; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t nuc = i / (n - 1), L = i - nuc * (n - 1);
+        const double *lo = pts + (nuc * n + L) * 6, *hi = lo + 6;
+        double *o = iv + i * 12;
+        o[0] = hi[0];
+        o[1] = __dsub_rn(hi[0], lo[0]);
+#pragma unroll
+        for (int c = 0; c < 5; c++) {
+            o[2 + 2 * c] = hi[1 + c];
+            o[3 + 2 * c] = __dsub_rn(hi[1 + c], lo[1 + c]);
+        }
+    }
+}
+
 __global__ void k_layout(int64_t N, int32_t n, const double *__restrict__ keys, const uint32_t *__restrict__ vals,
                          const double *__restrict__ raw, double *__restrict__ E, double *__restrict__ pts,
                          int *__restrict__ dup)
@@ -263,6 +280,12 @@ void build_grid(Grid &g)
                                                              (int)N, (int)g.n_nuc, offs, offs + 1));
         k_layout<<<grid_blocks(N, tpb), tpb>>>(N, n, keys_out, vals_out, raw, g.E, g.pts, dup);
         XS_CUDA_TRY(cudaGetLastError());
+        if (kIv) {
+            const int64_t NI = g.n_nuc * (n - 1);
+            g.iv = dalloc<double>(g, NI * 12);
+            k_iv_build<<<grid_blocks(NI, tpb), tpb>>>(NI, n, g.pts, g.iv);
+            XS_CUDA_TRY(cudaGetLastError());
+        }
         int dup_h = 0;
         XS_CUDA_TRY(cudaMemcpy(&dup_h, dup, sizeof(int), cudaMemcpyDeviceToHost));
         if (dup_h)
@@ -302,6 +325,17 @@ void build_grid(Grid &g)
             int b_log2 = 1;
             while ((int64_t(1) << b_log2) < g.n && b_log2 < 20)
                 b_log2++;
+            // oversample (up to 4x) while the point records and the bin table still fit in
+            // L2 together: fewer bins hold >= 2 points, so fewer pairs need a window probe
+            // (small tables 1.045x; large tables, already past L2, keep 2^k >= n)
+            int l2_bytes = 0;
+            XS_CUDA_TRY(cudaDeviceGetAttribute(&l2_bytes, cudaDevAttrL2CacheSize, g.device));
+            for (int extra = 0; extra < 2 && b_log2 < 22; extra++) {
+                const int64_t bytes = g.N * 48 + g.n_nuc * (int64_t)sizeof(BinEntry) * (int64_t(1) << (b_log2 + 1));
+                if (bytes > (int64_t)l2_bytes)
+                    break;
+                b_log2++;
+            }
             const int64_t per = int64_t(1) << b_log2;
             if (g.n_nuc * per < (int64_t(1) << 31)) {
                 g.b_log2 = b_log2;
@@ -365,7 +399,7 @@ void build_grid(Grid &g)
                 const int64_t nuc = mats[(size_t)m * g.max_nucs + j];
                 NucRef &r = refs[(size_t)m * g.max_nucs + j];
                 r.E = g.E + nuc * g.n;
-                r.pts = g.pts + nuc * g.n * 6;
+                r.pts = kIv ? g.iv + nuc * (g.n - 1) * 12 : g.pts + nuc * g.n * 6;
                 r.T = g.tkeys ? g.tkeys + nuc * g.t_per_nuc : nullptr;
                 r.B = g.bnd ? g.bnd + nuc * (int64_t(1) << g.b_log2) : nullptr;
                 r.conc = concs[(size_t)m * g.max_nucs + j];
@@ -385,6 +419,7 @@ void free_grid(Grid &g)
 {
     cudaFree(g.E);
     cudaFree(g.pts);
+    cudaFree(g.iv);
     cudaFree(g.tkeys);
     cudaFree(g.bnd);
     cudaFree(g.ubnd);
@@ -453,6 +488,7 @@ GridView make_view(const Grid &g)
     GridView v{};
     v.E = g.E;
     v.pts = g.pts;
+    v.iv = g.iv;
     v.U = g.U;
     v.IDX = g.IDX;
     v.H = g.H;

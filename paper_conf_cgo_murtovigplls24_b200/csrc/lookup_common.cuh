@@ -133,7 +133,7 @@ __device__ __forceinline__ Row make_row(const GridView &gv, int nuc)
 {
     Row r;
     r.E = opaque(gv.E + (size_t)nuc * (uint32_t)gv.n);
-    r.pts = gv.pts + (size_t)nuc * (uint32_t)gv.n * 6;
+    r.pts = kIv ? gv.iv + (size_t)nuc * (uint32_t)(gv.n - 1) * 12 : gv.pts + (size_t)nuc * (uint32_t)gv.n * 6;
     r.T = gv.tkeys ? gv.tkeys + (size_t)nuc * (uint32_t)gv.t_per_nuc : nullptr;
     r.B = gv.bnd ? gv.bnd + ((size_t)nuc << gv.b_log2) : nullptr;
     r.conc = 0.0;
@@ -244,6 +244,48 @@ struct Acc {
     double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0, a4 = 0.0;
 };
 
+// The interpolation of one pair (reading R8): f = (E_hi - q) / (E_hi - E_lo) by IEEE
+// division, micro_c = fma(-f, X_hi - X_lo, X_hi), acc_c = fma(micro_c, conc, acc_c).
+#if XS_IV
+// 96 B gather of interval L's record {E_hi, dE, (X_hi, dX) x 5}: six 16 B loads; dE and dX
+// were rounded at build time exactly as below, so the results are bit-identical
+__device__ __forceinline__ void accumulate_pair(const double *__restrict__ iv_row, int L, double q, double conc,
+                                                Acc &A)
+{
+    const double2 *p = reinterpret_cast<const double2 *>(iv_row) + (uint32_t)L * 6;
+    const double2 e = __ldg(p + 0), c0 = __ldg(p + 1), c1 = __ldg(p + 2);
+    const double2 c2 = __ldg(p + 3), c3 = __ldg(p + 4), c4 = __ldg(p + 5);
+    const double f = __ddiv_rn(__dsub_rn(e.x, q), e.y);
+    A.a0 = __fma_rn(__fma_rn(-f, c0.y, c0.x), conc, A.a0);
+    A.a1 = __fma_rn(__fma_rn(-f, c1.y, c1.x), conc, A.a1);
+    A.a2 = __fma_rn(__fma_rn(-f, c2.y, c2.x), conc, A.a2);
+    A.a3 = __fma_rn(__fma_rn(-f, c3.y, c3.x), conc, A.a3);
+    A.a4 = __fma_rn(__fma_rn(-f, c4.y, c4.x), conc, A.a4);
+}
+
+__device__ __forceinline__ void accumulate_pair2(const double *__restrict__ pa, int La, double ca,
+                                                 const double *__restrict__ pb, int Lb, double cb, double q, Acc &A)
+{
+    const double2 *p = reinterpret_cast<const double2 *>(pa) + (uint32_t)La * 6;
+    const double2 *s = reinterpret_cast<const double2 *>(pb) + (uint32_t)Lb * 6;
+    const double2 e = __ldg(p + 0), c0 = __ldg(p + 1), c1 = __ldg(p + 2);
+    const double2 c2 = __ldg(p + 3), c3 = __ldg(p + 4), c4 = __ldg(p + 5);
+    const double2 g = __ldg(s + 0), d0 = __ldg(s + 1), d1 = __ldg(s + 2);
+    const double2 d2 = __ldg(s + 3), d3 = __ldg(s + 4), d4 = __ldg(s + 5);
+    const double fa = __ddiv_rn(__dsub_rn(e.x, q), e.y);
+    const double fb = __ddiv_rn(__dsub_rn(g.x, q), g.y);
+    const double a0 = __fma_rn(-fa, c0.y, c0.x), b0 = __fma_rn(-fb, d0.y, d0.x);
+    const double a1 = __fma_rn(-fa, c1.y, c1.x), b1 = __fma_rn(-fb, d1.y, d1.x);
+    const double a2 = __fma_rn(-fa, c2.y, c2.x), b2 = __fma_rn(-fb, d2.y, d2.x);
+    const double a3 = __fma_rn(-fa, c3.y, c3.x), b3 = __fma_rn(-fb, d3.y, d3.x);
+    const double a4 = __fma_rn(-fa, c4.y, c4.x), b4 = __fma_rn(-fb, d4.y, d4.x);
+    A.a0 = __fma_rn(b0, cb, __fma_rn(a0, ca, A.a0));
+    A.a1 = __fma_rn(b1, cb, __fma_rn(a1, ca, A.a1));
+    A.a2 = __fma_rn(b2, cb, __fma_rn(a2, ca, A.a2));
+    A.a3 = __fma_rn(b3, cb, __fma_rn(a3, ca, A.a3));
+    A.a4 = __fma_rn(b4, cb, __fma_rn(a4, ca, A.a4));
+}
+#else
 // 96 B gather: the 48 B records of points L and L+1, three 16 B loads each
 __device__ __forceinline__ void accumulate_pair(const double *__restrict__ pts_row, int L, double q, double conc,
                                                 Acc &A)
@@ -283,6 +325,8 @@ __device__ __forceinline__ void accumulate_pair2(const double *__restrict__ pa, 
     A.a3 = __fma_rn(b3, cb, __fma_rn(a3, ca, A.a3));
     A.a4 = __fma_rn(b4, cb, __fma_rn(a4, ca, A.a4));
 }
+
+#endif
 
 // verification value (R10): 1 + first maximum, strict '>' from -1.0
 __device__ __forceinline__ uint32_t verify(const Acc &A)

@@ -33,6 +33,11 @@ void clear_error();
 
 constexpr int kMaterials = 12;
 constexpr int kMaxEnergyBins = 4096;
+#ifndef XS_IV
+#define XS_IV 0
+#endif
+// XS_IV: lookups interpolate from per-interval records (iv) instead of point pairs (pts)
+constexpr bool kIv = XS_IV;
 constexpr int kTreeFan = 16;     // separator keys per node: one 128 B line
 constexpr int kTreeMaxLevels = 6; // n < 17^6 * 16 for every n_gridpoints < 2^31
 
@@ -56,6 +61,10 @@ struct Grid {
 
     double *E = nullptr;
     double *pts = nullptr;
+    // iv [n_nuc][n-1][12]: interval L's record {E[L+1], E[L+1]-E[L], (X_c[L+1],
+    // X_c[L+1]-X_c[L]) for c = 0..4} -- the differences the interpolation needs, rounded
+    // once at build time exactly as the lookup would round them (XS_IV)
+    double *iv = nullptr;
     // separator tree of every nuclide row (XS_SEARCH_W): level d has
     // 17^d nodes of 16 keys; node keys are E at base + (t+1)*stride[d] (+inf past n)
     double *tkeys = nullptr;
@@ -126,7 +135,8 @@ struct alignas(16) BinEntry {
 // creation so the loop does one 32 B broadcast load instead of 64-bit row arithmetic.
 struct NucRef {
     const double *E;   // energy row of the nuclide            (E + nuc * n)
-    const double *pts; // 48 B point records of the nuclide    (pts + nuc * n * 6)
+    const double *pts; // interpolation records: pts + nuc*n*6 (48 B points) or, with XS_IV,
+                       // iv + nuc*(n-1)*12 (96 B intervals)
     const double *T;   // separator tree of the nuclide, or NULL
     const BinEntry *B; // bin table of the nuclide, or NULL
     double conc;       // concs[m][j]
@@ -136,6 +146,7 @@ struct NucRef {
 struct GridView {
     const double *__restrict__ E;
     const double *__restrict__ pts;
+    const double *__restrict__ iv;
     const double *__restrict__ U;
     const int32_t *__restrict__ IDX;
     const int32_t *__restrict__ H;
