@@ -14,7 +14,12 @@ HEADER = os.path.join(ROOT, "include", "xs.h")
 
 @pytest.fixture(scope="module")
 def xs():
-    from paper_conf_cgo_murtovigplls24_b200 import build
+    import importlib.util
+    # by path: the package's __init__ refuses to import before libxs.so exists
+    spec = importlib.util.spec_from_file_location(
+        "_xs_build", os.path.join(ROOT, "paper_conf_cgo_murtovigplls24_b200", "build.py"))
+    build = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(build)
     build.build()
     import paper_conf_cgo_murtovigplls24_b200 as pkg
     return pkg
