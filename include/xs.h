@@ -72,7 +72,15 @@ enum {
                          grid idea (R7) at power-of-two resolution.  On the unionized grid
                          the same table over U bounds the one U search per lookup; on the
                          hash grid (whose 10,000-bin table is the configuration) it is U2. */
-    XS_SEARCH_COUNT = 11
+    XS_SEARCH_S = 11, /* staged warp window (sorted modes): a warp whose
+                         lookups share a material takes q_min, q_max over its lanes; lane t
+                         finds [L(q_min), L(q_max)] of nuclide t (H bounds) and copies that
+                         window's point records into shared memory, 32 nuclides at a time;
+                         each lane then runs Listing 1 (U1) on the staged window energies
+                         and interpolates from shared memory.  L(q) is exact because L is
+                         monotone in q.  Windows that do not fit, mixed-material warps and
+                         unsorted lookups take the H path.                               */
+    XS_SEARCH_COUNT = 12
 };
 
 /* Lookup ordering (a pure reordering: results are invariant). */

@@ -10,7 +10,7 @@ from __future__ import annotations
 from ._xs import (  # noqa: F401  (the C names)
     SEARCH_NAMES, SORT_NAMES, XS_ECUDA, XS_EDUP, XS_EINVAL, XS_ENOMEM, XS_FLAG_SPLIT, XS_FLAG_TIMING, XS_HASH, XS_NUCLIDE, XS_OK,
     XS_SEARCH_B, XS_SEARCH_COUNT, XS_SEARCH_M, XS_SEARCH_M2, XS_SEARCH_M4, XS_SEARCH_M8, XS_SEARCH_U1,
-    XS_SEARCH_U2, XS_SEARCH_U4, XS_SEARCH_U8, XS_SEARCH_W, XS_SEARCH_H, XS_SORT_HISTORY, XS_SORT_MATERIAL, XS_SORT_MATERIAL_ENERGY, XS_SORT_NONE,
+    XS_SEARCH_U2, XS_SEARCH_U4, XS_SEARCH_U8, XS_SEARCH_W, XS_SEARCH_H, XS_SEARCH_S, XS_SORT_HISTORY, XS_SORT_MATERIAL, XS_SORT_MATERIAL_ENERGY, XS_SORT_NONE,
     XS_UNIONIZED, LIB_PATH, XSError, xs_grid_checksum, xs_grid_create, xs_grid_destroy, xs_grid_export,
     xs_grid_export_aux, xs_grid_get_info, xs_last_error, xs_lookup_batch, xs_lookup_indices, xs_lookup_range,
     xs_opts, xs_opts_default, xs_sample, xs_search_points, xs_stats,

@@ -27,13 +27,13 @@ _lib = C.CDLL(LIB_PATH)
 XS_UNIONIZED, XS_NUCLIDE, XS_HASH = 0, 1, 2
 XS_OK, XS_EINVAL, XS_ENOMEM, XS_ECUDA, XS_EDUP = 0, -1, -2, -3, -4
 (XS_SEARCH_M, XS_SEARCH_U1, XS_SEARCH_U2, XS_SEARCH_U4, XS_SEARCH_U8, XS_SEARCH_B,
- XS_SEARCH_M2, XS_SEARCH_M4, XS_SEARCH_M8, XS_SEARCH_W, XS_SEARCH_H) = range(11)
-XS_SEARCH_COUNT = 11
+ XS_SEARCH_M2, XS_SEARCH_M4, XS_SEARCH_M8, XS_SEARCH_W, XS_SEARCH_H, XS_SEARCH_S) = range(12)
+XS_SEARCH_COUNT = 12
 XS_SORT_NONE, XS_SORT_MATERIAL, XS_SORT_MATERIAL_ENERGY, XS_SORT_HISTORY = 0, 1, 2, 3
 XS_FLAG_TIMING = 1
 XS_FLAG_SPLIT = 2
 
-SEARCH_NAMES = {"M": 0, "U1": 1, "U2": 2, "U4": 3, "U8": 4, "B": 5, "M2": 6, "M4": 7, "M8": 8, "W": 9, "H": 10}
+SEARCH_NAMES = {"M": 0, "U1": 1, "U2": 2, "U4": 3, "U8": 4, "B": 5, "M2": 6, "M4": 7, "M8": 8, "W": 9, "H": 10, "S": 11}
 SORT_NAMES = {"none": 0, "material": 1, "material_energy": 2, "history": 3}
 XS_BZ_M, XS_BZ_M2, XS_BZ_U1, XS_BZ_U2, XS_BZ_S, XS_BZ_T = range(6)
 XS_BZ_COUNT = 6

@@ -147,7 +147,7 @@ __device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, do
 {
     const double *__restrict__ Ei = rw.E;
     const int nuc = rw.nuc;
-    if constexpr (GRID == XS_NUCLIDE && SEARCH == XS_SEARCH_H) {
+    if constexpr (GRID == XS_NUCLIDE && (SEARCH == XS_SEARCH_H || SEARCH == XS_SEARCH_S)) {
         // bin-bounded window
         if (gv.b_log2 > 0 && q >= 0.0 && q <= 1.0)
             return bin_lower(Ei, load_bin(rw.B + bin_of(q, gv.b_log2)), q);
@@ -170,7 +170,7 @@ __device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, do
 template <int GRID, int SEARCH>
 __device__ __forceinline__ int union_index(const GridView &gv, double q)
 {
-    if constexpr (GRID == XS_UNIONIZED && SEARCH == XS_SEARCH_H) {
+    if constexpr (GRID == XS_UNIONIZED && (SEARCH == XS_SEARCH_H || SEARCH == XS_SEARCH_S)) {
         // the same bin-bounded window over the unionized energies (R4 + §6.5)
         if (gv.u_log2 > 0 && q >= 0.0 && q <= 1.0)
             return bin_lower(opaque(gv.U), load_bin(gv.ubnd + bin_of(q, gv.u_log2)), q);

@@ -357,6 +357,10 @@ void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, c
                  : k_lookup<XS_NUCLIDE, XS_SEARCH_H, true, false, true>;
         blocks = std::min(blocks, blocks / 4 * 3 > 0 ? blocks / 4 * 3 : blocks); // one wave at 3 CTAs/SM
     }
+    if (search == XS_SEARCH_S && sorted) { // the staged-window kernel (lookup_staged.cu)
+        launch_staged(grid_type, blocks, tpb, stream, gv, sv, so, out, out_idx, stats);
+        return;
+    }
     f<<<blocks, tpb, 0, stream>>>(gv, sv, so, J_grid, out, out_idx, stats);
     XS_CUDA_TRY(cudaGetLastError());
 }

@@ -1,0 +1,362 @@
+// lookup_staged.cu -- XS_SEARCH_S: the sorted lookup kernel with staged warp windows
+// (DESIGN.md §6.5c).  Same work queue as k_lookup (lookup_fused.cu): each warp pulls chunks
+// of 4 x 32 consecutive sorted slots.  Per iteration a warp takes 32 lookups; for each
+// material among them (in sorted order almost always one) the lanes of that material form
+// the window [q_lo, q_hi] and every nuclide of the material is resolved through a window
+// of interval records staged in shared memory.
+#include <algorithm>
+
+#include "lookup_common.cuh"
+
+namespace xs {
+
+constexpr int kStTpb = 256;
+#ifndef XS_S_MIN_BLOCKS
+#define XS_S_MIN_BLOCKS 3
+#endif
+#ifndef XS_S_CHUNK
+#define XS_S_CHUNK 128
+#endif
+constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pulls one at a time)
+#ifndef XS_S_LPL
+#define XS_S_LPL 2
+#endif
+constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the staged windows
+
+// ---- XS_SEARCH_S: staged warp windows -----------------------------------
+// Per warp in dynamic shared memory: kStageCap interval records, their upper energies again
+// in a compact array (the window count reads them), 32 window descriptors and the owner
+// lane of every staged interval.  Interval record (112 B = 7 x 16 B): the quantities of
+// reading R8 that do not depend on q, rounded exactly as accumulate_pair rounds them,
+//   [0] E_hi  [1] d = E_hi - E_lo  [2] y = RN(1/d)  [3 + 2c] X_c,hi  [4 + 2c] dX_c = X_c,hi - X_c,lo
+// so a pair costs one subtraction, Markstein's quotient (3 ops) and 10 FMAs.
+#ifndef XS_STAGE_CAP
+#define XS_STAGE_CAP 48
+#endif
+constexpr int kStageCap = XS_STAGE_CAP; // intervals per warp
+constexpr int kIvDoubles = 14;
+struct alignas(16) StageMeta {
+    double conc;
+    int32_t lo;     // L(q_min) of the nuclide
+    int32_t offcnt; // (first staged interval << 16) | intervals, or -1: not staged
+};
+constexpr int kStageWarpBytes =
+    kStageCap * kIvDoubles * 8 + kStageCap * 8 + 32 * (int)sizeof(StageMeta) + ((kStageCap + 15) / 16) * 16;
+
+struct WarpStage {
+    double *rec;     // [kStageCap][kIvDoubles]
+    double *eh;      // [kStageCap] E_hi of each staged interval
+    StageMeta *meta; // [32]
+    uint8_t *owner;  // [kStageCap]
+};
+
+__device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
+{
+    WarpStage w;
+    unsigned char *base = smem + (threadIdx.x >> 5) * kStageWarpBytes;
+    w.rec = reinterpret_cast<double *>(base);
+    w.eh = w.rec + kStageCap * kIvDoubles;
+    w.meta = reinterpret_cast<StageMeta *>(w.eh + kStageCap);
+    w.owner = reinterpret_cast<uint8_t *>(w.meta + 32);
+    return w;
+}
+
+// f = RN(a / d) from y = RN(1/d): q0 = RN(a y), r = a - d q0 (exact, an FMA), f = RN(q0 + r y).
+// Markstein's theorem: with y within half an ulp of 1/d and q0 within one ulp of a/d (both
+// hold here, and a, d are far from under/overflow: multiples of 2^-63 in (-1, 1)), f is the
+// correctly rounded quotient, i.e. bit-identical to IEEE division (__ddiv_rn); pinned on the
+// CPU by tests/test_markstein.py, and by every bit-exact parity test of XS_SEARCH_S.
+__device__ __forceinline__ double quotient_markstein(double a, double d, double y)
+{
+    const double q0 = __dmul_rn(a, y);
+    const double r = __fma_rn(-d, q0, a);
+    return __fma_rn(r, y, q0);
+}
+
+// the interpolation of accumulate_pair (reading R8; identical results) from a staged
+// interval record
+__device__ __forceinline__ void accumulate_interval(const double *R, double q, double conc, Acc &A)
+{
+    const double2 *p = reinterpret_cast<const double2 *>(R);
+    const double2 e = p[0], x0 = p[1], x1 = p[2], x2 = p[3], x3 = p[4], x4 = p[5], x5 = p[6];
+    const double f = quotient_markstein(__dsub_rn(e.x, q), e.y, x0.x);
+    A.a0 = __fma_rn(__fma_rn(-f, x1.x, x0.y), conc, A.a0);
+    A.a1 = __fma_rn(__fma_rn(-f, x2.x, x1.y), conc, A.a1);
+    A.a2 = __fma_rn(__fma_rn(-f, x3.x, x2.y), conc, A.a2);
+    A.a3 = __fma_rn(__fma_rn(-f, x4.x, x3.y), conc, A.a3);
+    A.a4 = __fma_rn(__fma_rn(-f, x5.x, x4.y), conc, A.a4);
+}
+
+// interval record k of a point row (points k and k+1) into shared memory
+__device__ __forceinline__ void stage_interval(const double *__restrict__ pts, int k, double *dst, double *eh)
+{
+    const double2 *p = reinterpret_cast<const double2 *>(pts) + (size_t)(uint32_t)k * 3;
+    const double2 a0 = __ldg(p), a1 = __ldg(p + 1), a2 = __ldg(p + 2);
+    const double2 b0 = __ldg(p + 3), b1 = __ldg(p + 4), b2 = __ldg(p + 5);
+    const double d = __dsub_rn(b0.x, a0.x);
+    double2 *o = reinterpret_cast<double2 *>(dst);
+    o[0] = make_double2(b0.x, d);
+    o[1] = make_double2(__drcp_rn(d), b0.y);
+    o[2] = make_double2(__dsub_rn(b0.y, a0.y), b1.x);
+    o[3] = make_double2(__dsub_rn(b1.x, a1.x), b1.y);
+    o[4] = make_double2(__dsub_rn(b1.y, a1.y), b2.x);
+    o[5] = make_double2(__dsub_rn(b2.x, a2.x), b2.y);
+    o[6] = make_double2(__dsub_rn(b2.y, a2.y), 0.0);
+    *eh = b0.x;
+}
+
+// c = #{k in 1..cnt-1 : E[lo + k] <= q} (E[lo + k] = eh[k - 1]), i.e. L(q) - lo: short
+// windows by three compares of values shared by the lane's lookups, longer ones by Listing 1
+// (U1) over eh
+__device__ __forceinline__ int window_count(const double *eh, int cnt, double q)
+{
+    int c = 0, len = cnt;
+    while (len > 1) {
+        const int h = len >> 1;
+        if (eh[c + h - 1] > q) {
+            len = h;
+        } else {
+            c += h;
+            len -= h;
+        }
+    }
+    return c;
+}
+
+// The lookups in `mine` (one material: row `roww`, nn nuclides; kLpl per lane) accumulate
+// every nuclide of the material.  All 32 lanes call it (warp collectives inside).
+template <int GRID, bool OUTS>
+__device__ __forceinline__ void staged_material(const GridView &gv, int roww, int nn, const bool (&mine)[kLpl],
+                                                const double (&q)[kLpl], const uint32_t (&r)[kLpl],
+                                                const WarpStage &ws, int32_t *__restrict__ out_idx,
+                                                Acc (&A)[kLpl])
+{
+    const int lane = threadIdx.x & 31;
+    // every lookup of the material has q in [q_lo, q_hi] and L is monotone, so
+    // L(q) = L(q_lo) + #{k in (L(q_lo), L(q_hi)] : E[k] <= q}
+    double mn = __longlong_as_double(0x7FF0000000000000ll), mx = -1.0;
+#pragma unroll
+    for (int l = 0; l < kLpl; l++) {
+        mn = mine[l] ? fmin(mn, q[l]) : mn;
+        mx = mine[l] ? fmax(mx, q[l]) : mx;
+    }
+    const double q_lo = warp_min(mn), q_hi = warp_max(mx);
+    int e_lo = 0, e_hi = 0;
+    if constexpr (GRID == XS_UNIONIZED) {
+        e_lo = union_index<GRID, XS_SEARCH_S>(gv, q_lo);
+        e_hi = union_index<GRID, XS_SEARCH_S>(gv, q_hi);
+    }
+    for (int g0 = 0; g0 < nn; g0 += 32) {
+        // lane t: the window of nuclide g0 + t (H bounds), intervals lo .. lo + cnt - 1
+        const int ng = min(32, nn - g0);
+        int lo = 0, cnt = 0;
+        double conc = 0.0;
+        const double *pts = nullptr;
+        if (lane < ng) {
+            const Row rw = load_row(gv, roww + g0 + lane);
+            lo = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_lo, e_lo);
+            cnt = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_hi, e_hi) - lo + 1;
+            conc = rw.conc;
+            pts = rw.pts;
+        }
+        for (int b0 = 0; b0 < ng;) { // passes over the group (warp-uniform)
+            const int want = (lane >= b0) ? cnt : 0;
+            int incl = want;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(0xffffffffu, incl, o);
+                incl += (lane >= o) ? t : 0;
+            }
+            const bool fits = want > 0 && incl <= kStageCap; // lanes b0 .. b1-1
+            const int nfit = __popc(__ballot_sync(0xffffffffu, fits));
+            const int T = nfit ? __shfl_sync(0xffffffffu, incl, b0 + nfit - 1) : 0; // intervals staged
+            int b1 = b0 + nfit;
+            const int off = incl - want;
+            __syncwarp(); // the previous pass's shared-memory reads are done
+            if (fits) {
+                ws.meta[lane] = StageMeta{conc, lo, (off << 16) | cnt};
+                for (int k = 0; k < cnt; k++)
+                    ws.owner[off + k] = (uint8_t)lane;
+            }
+            if (b1 == b0) { // nuclide b0's window alone exceeds the stage: per-lane H path
+                if (lane == b0)
+                    ws.meta[lane] = StageMeta{conc, lo, -1};
+                b1 = b0 + 1;
+            }
+            __syncwarp();
+            // interval i of the pass is staged by lane i % 32: owner nuclide j, its k-th interval
+            for (int i0 = 0; i0 < T; i0 += 32) {
+                const int i = i0 + lane;
+                const int j = i < T ? ws.owner[i] : b0;
+                const double *pj = reinterpret_cast<const double *>(
+                    __shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(pts), j));
+                const int lo_j = __shfl_sync(0xffffffffu, lo, j);
+                const int off_j = __shfl_sync(0xffffffffu, off, j);
+                if (i < T)
+                    stage_interval(pj, lo_j + (i - off_j), ws.rec + i * kIvDoubles, ws.eh + i);
+            }
+            __syncwarp();
+            for (int jj = b0; jj < b1; jj++) { // ascending nuclide order (R8)
+                const StageMeta m = ws.meta[jj];
+                if (m.offcnt >= 0) {
+                    const int off_w = m.offcnt >> 16, cnt_w = m.offcnt & 0xFFFF;
+                    const double *eh = ws.eh + off_w;
+                    const double *R = ws.rec + off_w * kIvDoubles;
+                    if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
+                        const double inf = __longlong_as_double(0x7FF0000000000000ll);
+                        const double e1 = cnt_w > 1 ? eh[0] : inf;
+                        const double e2 = cnt_w > 2 ? eh[1] : inf;
+                        const double e3 = cnt_w > 3 ? eh[2] : inf;
+#pragma unroll
+                        for (int l = 0; l < kLpl; l++) {
+                            if (mine[l]) {
+                                const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
+                                accumulate_interval(R + c * kIvDoubles, q[l], m.conc, A[l]);
+                                if constexpr (OUTS) {
+                                    if (out_idx)
+                                        out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo + c;
+                                }
+                            }
+                        }
+                    } else {
+#pragma unroll
+                        for (int l = 0; l < kLpl; l++) {
+                            if (mine[l]) {
+                                const int c = window_count(eh, cnt_w, q[l]);
+                                accumulate_interval(R + c * kIvDoubles, q[l], m.conc, A[l]);
+                                if constexpr (OUTS) {
+                                    if (out_idx)
+                                        out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo + c;
+                                }
+                            }
+                        }
+                    }
+                } else {
+                    const Row rw = load_row(gv, roww + g0 + jj);
+#pragma unroll
+                    for (int l = 0; l < kLpl; l++) {
+                        if (mine[l]) {
+                            int e_me = 0;
+                            if constexpr (GRID == XS_UNIONIZED)
+                                e_me = union_index<GRID, XS_SEARCH_S>(gv, q[l]);
+                            const int L = lower_index<GRID, XS_SEARCH_S>(gv, rw, q[l], e_me);
+                            accumulate_pair(rw.pts, L, q[l], rw.conc, A[l]);
+                            if constexpr (OUTS) {
+                                if (out_idx)
+                                    out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = L;
+                            }
+                        }
+                    }
+                }
+            }
+            b0 = b1;
+        }
+    }
+}
+
+template <int GRID, bool OUTS>
+__global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
+    k_lookup_staged(GridView gv, SortedView so, int count, double *__restrict__ out_, int32_t *__restrict__ out_idx_,
+                    unsigned long long *__restrict__ stats)
+{
+    double *__restrict__ out = OUTS ? out_ : nullptr;
+    int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
+    extern __shared__ __align__(16) unsigned char st_smem[];
+    __shared__ uint32_t s_mb[kMaterials + 1];
+    if (threadIdx.x <= kMaterials)
+        s_mb[threadIdx.x] = __ldg(so.mb_dev + threadIdx.x);
+    __syncthreads();
+    const WarpStage ws = warp_stage(st_smem);
+    const int lane = threadIdx.x & 31;
+    const uint64_t pol = policy_evict_first();
+    uint32_t my_hash = 0, my_pairs = 0;
+    for (;;) {
+        int c;
+        if (lane == 0)
+            c = atomicAdd(so.work, 1);
+        c = __shfl_sync(0xffffffffu, c, 0);
+        if (c * kStChunk >= count)
+            break;
+        const int jend = min(count, c * kStChunk + kStChunk);
+        for (int jw = c * kStChunk; jw < jend; jw += 32 * kLpl) {
+            bool act[kLpl], mine[kLpl];
+            double q[kLpl];
+            uint32_t r[kLpl];
+            int mat[kLpl];
+            Acc A[kLpl];
+            unsigned todo[kLpl];
+#pragma unroll
+            for (int l = 0; l < kLpl; l++) {
+                const int j = jw + l * 32 + lane;
+                act[l] = j < jend;
+                r[l] = act[l] ? ld_stream(so.slot + j, pol) : 0u;
+                q[l] = act[l] ? ld_stream(so.q_of + r[l], pol) : 0.0;
+                mat[l] = act[l] ? material_of(s_mb, (uint32_t)j) : 0;
+                todo[l] = __ballot_sync(0xffffffffu, act[l]);
+            }
+            // one round per material among the warp's lookups (sorted: almost always one)
+            for (;;) {
+                int src = -1;
+#pragma unroll
+                for (int l = kLpl - 1; l >= 0; l--)
+                    src = todo[l] ? l * 32 + __ffs(todo[l]) - 1 : src;
+                if (src < 0)
+                    break;
+                int mw = mat[0];
+#pragma unroll
+                for (int l = 1; l < kLpl; l++)
+                    mw = (src >> 5) == l ? mat[l] : mw;
+                const int mat_w = __shfl_sync(0xffffffffu, mw, src & 31);
+#pragma unroll
+                for (int l = 0; l < kLpl; l++) {
+                    mine[l] = act[l] && mat[l] == mat_w;
+                    todo[l] &= ~__ballot_sync(0xffffffffu, mine[l]);
+                }
+                staged_material<GRID, OUTS>(gv, mat_w * gv.max_nucs, __ldg(gv.num_nucs + mat_w), mine, q, r, ws,
+                                            out_idx, A);
+            }
+#pragma unroll
+            for (int l = 0; l < kLpl; l++) {
+                if (act[l]) {
+                    my_hash += verify(A[l]);
+                    my_pairs += (uint32_t)__ldg(gv.num_nucs + mat[l]);
+                    if (out)
+                        store_macro(out, r[l], A[l]);
+                }
+            }
+        }
+    }
+    reduce_stats<kStTpb>(my_hash, my_pairs, stats);
+}
+
+using StagedFn = void (*)(GridView, SortedView, int, double *, int32_t *, unsigned long long *);
+
+template <int GRID> static StagedFn pick_staged(bool outs)
+{
+    return outs ? k_lookup_staged<GRID, true> : k_lookup_staged<GRID, false>;
+}
+
+void launch_staged(int grid_type, int blocks, int tpb, cudaStream_t stream, const GridView &gv,
+                   const SampleView &sv, const SortedView &so, double *out, int32_t *out_idx,
+                   unsigned long long *stats)
+{
+    const bool outs = out || out_idx;
+    StagedFn f = grid_type == XS_NUCLIDE     ? pick_staged<XS_NUCLIDE>(outs)
+                 : grid_type == XS_UNIONIZED ? pick_staged<XS_UNIONIZED>(outs)
+                                             : pick_staged<XS_HASH>(outs);
+    (void)tpb; // one configuration: 256 threads, XS_S_MIN_BLOCKS CTAs per SM
+    const int smem = (kStTpb / 32) * kStageWarpBytes;
+    XS_CUDA_TRY(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    int per_sm = 0;
+    XS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, kStTpb, smem));
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int want = (int)((sv.count + kStTpb - 1) / kStTpb);
+    const int nb = std::max(1, std::min(want, sms * std::max(per_sm, 1)));
+    (void)blocks;
+    f<<<nb, kStTpb, smem, stream>>>(gv, so, (int)sv.count, out, out_idx, stats);
+    XS_CUDA_TRY(cudaGetLastError());
+}
+
+} // namespace xs

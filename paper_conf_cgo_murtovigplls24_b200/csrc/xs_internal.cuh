@@ -216,6 +216,11 @@ void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, c
                   const GridView &gv, const SampleView &sv, const SortedView &so, Affine J_grid, double *out,
                   int32_t *out_idx, unsigned long long *stats);
 
+// lookup_staged.cu: XS_SEARCH_S in sorted order (one persistent wave, 256 threads per CTA)
+void launch_staged(int grid_type, int blocks, int tpb, cudaStream_t stream, const GridView &gv,
+                   const SampleView &sv, const SortedView &so, double *out, int32_t *out_idx,
+                   unsigned long long *stats);
+
 // lookup_fused.cu: XSBench history order (XS_SORT_HISTORY)
 void launch_history(int grid_type, int search, int hl, int blocks, cudaStream_t stream, const GridView &gv,
                     const SampleView &sv, double *out, int32_t *out_idx, unsigned long long *stats);

@@ -19,7 +19,7 @@ first, count = 777, 23_456
 ref = P.run_range(1070, first, count, idx=True)
 with xs.Grid(68, 1000, 1, 42) as g:
     for sort, split in (("none", False), ("material_energy", False), ("material_energy", True), ("history", False)):
-        for search in ("M", "U2", "W", "H"):
+        for search in ("M", "U2", "W", "H", "S"):
             out, st = g.macro_xs(first, count, 1070, search=search, sort=sort, split=split, history_len=34)
             assert st.hash == ref["hash"] and st.pairs == ref["pairs"], (sort, split, search)
             assert np.array_equal(out.cpu().numpy(), ref["macro"]), (sort, split, search)

@@ -13,7 +13,7 @@ pytestmark = pytest.mark.gpu
 
 from xs_workloads import GRID_SEED, LOOKUP_SEED, WORKLOADS  # noqa: E402
 
-SEARCHES = ["M", "U1", "U2", "U4", "U8", "B", "M2", "M4", "M8", "W", "H"]
+SEARCHES = ["M", "U1", "U2", "U4", "U8", "B", "M2", "M4", "M8", "W", "H", "S"]
 SORTS = ["none", "material", "material_energy"]
 RTOL = 1e-12
 
@@ -115,9 +115,13 @@ def test_tiny_macro_and_hash(tiny, gt, search, sort, split):
 # ------------------------------------------------------------------ edge cases
 @pytest.mark.parametrize("first,count", [(0, 0), (0, 1), (7, 31), (1000, 257), (99_000, 1000), (3, 4097)])
 @pytest.mark.parametrize("sort,split", PIPES)
-def test_ragged_ranges(tiny, first, count, sort, split):
-    g, P, ref = tiny[1]
-    out, st = g.macro_xs(first, count, LOOKUP_SEED, sort=sort, split=split)
+@pytest.mark.parametrize("search", ["H", "S"])
+@pytest.mark.parametrize("gt", [0, 1, 2])
+def test_ragged_ranges(tiny, first, count, sort, split, search, gt):
+    """partial warps / CTAs / chunks; S's staged path needs the warp's material from an
+    active lane (inactive lanes carry material 0)"""
+    g, P, ref = tiny[gt]
+    out, st = g.macro_xs(first, count, LOOKUP_SEED, sort=sort, split=split, search=search)
     r = P.run_range(LOOKUP_SEED, first, count)
     assert st.hash == r["hash"] and st.pairs == r["pairs"]
     assert np.array_equal(out.cpu().numpy(), r["macro"])
@@ -125,9 +129,12 @@ def test_ragged_ranges(tiny, first, count, sort, split):
 
 @pytest.mark.parametrize("bins", [1, 2, 64, 1024, 4096])
 @pytest.mark.parametrize("block", [64, 128, 256])
-def test_energy_bins_and_block(tiny, bins, block):
+@pytest.mark.parametrize("search", ["H", "S"])
+def test_energy_bins_and_block(tiny, bins, block, search):
+    """few energy bins = wide warp windows: S's stage overflows into its per-lane path"""
     g, P, ref = tiny[1]
-    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, sort="material_energy", energy_bins=bins, block=block)
+    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, sort="material_energy", energy_bins=bins, block=block,
+                         search=search)
     assert st.hash == ref["hash"]
     assert np.array_equal(out.cpu().numpy(), ref["macro"])
 
@@ -197,25 +204,32 @@ def test_determinism_and_shards(tiny):
 
 
 # ------------------------------------------------------------------ full-size configs
-def _sampled_check(g, P, n_total, search="U2", sort="material_energy", n_samples=2000, prefix=200_000):
-    """Full-size launch (the bench configuration) on device, then sampled outputs + a prefix hash."""
-    out = torch.empty((n_total, 5), dtype=torch.float64, device=g.device)
-    st = g.lookup_range(0, n_total, LOOKUP_SEED, out, search=search, sort=sort)
+def _sampled_check(g, P, n_total, searches=("U2", "H", "S"), sort="material_energy", n_samples=2000,
+                   prefix=200_000):
+    """Full-size launch (the bench configuration: H and S are the bench's searches) on device,
+    then sampled outputs + a prefix hash, for each search variant against one oracle sample."""
     rng = np.random.default_rng(1)
     idx = np.unique(np.concatenate([rng.integers(0, n_total, n_samples), [0, n_total - 1]]))
     _, ref_macro = P.run_indices(LOOKUP_SEED, idx)
-    got = out[torch.as_tensor(idx, device=g.device)].cpu().numpy()
-    assert _macro_close(got, ref_macro) <= RTOL
-    assert np.array_equal(got, ref_macro)
     ref_prefix = P.run_range(LOOKUP_SEED, 0, prefix, macro=False)
-    assert g.lookup_range(0, prefix, LOOKUP_SEED, search=search, sort=sort).hash == ref_prefix["hash"]
-    # hash properties that hold at any size
-    assert st.lookups == n_total and n_total <= st.hash <= 5 * n_total
-    # v = 1 + first argmax with XSBench's start value max = -1.0 (R10): prepend a -1.0
-    # column (extrapolated lookups, R6, can have every channel below -1.0)
-    aug = torch.cat([torch.full((n_total, 1), -1.0, dtype=out.dtype, device=out.device), out], dim=1)
-    v = torch.clamp(torch.argmax(aug, dim=1), min=1)
-    assert int(v.sum().item()) == st.hash
+    hashes = set()
+    for search in searches:
+        out = torch.empty((n_total, 5), dtype=torch.float64, device=g.device)
+        st = g.lookup_range(0, n_total, LOOKUP_SEED, out, search=search, sort=sort)
+        got = out[torch.as_tensor(idx, device=g.device)].cpu().numpy()
+        assert _macro_close(got, ref_macro) <= RTOL, search
+        assert np.array_equal(got, ref_macro), search
+        assert g.lookup_range(0, prefix, LOOKUP_SEED, search=search, sort=sort).hash == ref_prefix["hash"], search
+        # hash properties that hold at any size
+        assert st.lookups == n_total and n_total <= st.hash <= 5 * n_total
+        # v = 1 + first argmax with XSBench's start value max = -1.0 (R10): prepend a -1.0
+        # column (extrapolated lookups, R6, can have every channel below -1.0)
+        aug = torch.cat([torch.full((n_total, 1), -1.0, dtype=out.dtype, device=out.device), out], dim=1)
+        v = torch.clamp(torch.argmax(aug, dim=1), min=1)
+        assert int(v.sum().item()) == st.hash, search
+        hashes.add(st.hash)
+        del out, aug, v
+    assert len(hashes) == 1
     return st
 
 
@@ -224,7 +238,7 @@ def test_small_full_hash(xs, oracle_mod):
     g = xs.Grid(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
     P = oracle_mod.Problem(w.n_nuclides, w.n_gridpoints, 1, GRID_SEED)
     ref = P.run_range(LOOKUP_SEED, 0, w.lookups, macro=False)
-    for search in ("M", "U2", "U4"):
+    for search in ("M", "U2", "U4", "H", "S"):
         for split in (False, True):
             st = g.lookup_range(0, w.lookups, LOOKUP_SEED, search=search, split=split)
             assert st.hash == ref["hash"] and st.pairs == ref["pairs"]

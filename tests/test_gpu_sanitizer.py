@@ -16,7 +16,7 @@ import torch
 import paper_conf_cgo_murtovigplls24_b200 as xs
 for gt in (0, 1, 2):
     g = xs.Grid(68, 200, gt, 42)
-    for search in ("M", "U2", "W", "H"):
+    for search in ("M", "U2", "W", "H", "S"):
         for sort in ("none", "material_energy"):
             out, st = g.macro_xs(0, 3000, 1070, search=search, sort=sort)
     g.indices(5, 1000, 1070, sort="material_energy", split=True)
