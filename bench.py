@@ -47,13 +47,13 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="small", choices=sorted(WORKLOADS))
     p.add_argument("--lookups", type=int, default=0, help="override lookups per GPU")
-    p.add_argument("--search", default="H")
+    p.add_argument("--search", default="S")
     p.add_argument("--sort", default="material_energy")
     p.add_argument("--energy-bins", type=int, default=0)
     p.add_argument("--no-flush", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--ab", default="M,U1,U2,U4,U8,B,W,H", help="search variants for the A/B sub-object ('' = off)")
+    p.add_argument("--ab", default="M,U1,U2,U4,U8,B,W,H,S", help="search variants for the A/B sub-object ('' = off)")
     p.add_argument("--ab-steps", type=int, default=5)
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target wall time of the CPU sample")
     return p.parse_args()
@@ -329,7 +329,7 @@ def run_ours(a, w):
         "step_ms": {"median": statistics.median(step_ms), "rsd_pct": 100 * statistics.pstdev(step_ms) /
                     statistics.mean(step_ms), "min": min(step_ms), "max": max(step_ms)},
         "phase_ms": {"sort": statistics.mean(s.sample_ms for s in stats), "lookup": mean_lookup_ms},
-        "roofline": {"bound": "hbm", "kernel": "k_lookup", "achieved": achieved, "peak": peak, "unit": "GB/s",
+        "roofline": {"bound": "hbm", "kernel": "k_lookup_staged" if a.search == "S" and a.sort == "material_energy" else "k_lookup", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "bytes_per_lookup_alg": bpl, "peak_source": peak_src,
                      "note": "achieved = SURVEY.md §8d random-gather bytes (E[nuclides] x 96 B per lookup) / "

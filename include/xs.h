@@ -140,7 +140,7 @@ typedef struct xs_grid_info {
     int32_t num_nucs[12];
 } xs_grid_info;
 
-/* Fill *opts with the defaults: XS_SEARCH_H, XS_SORT_MATERIAL_ENERGY, legacy stream, no flags. */
+/* Fill *opts with the defaults: XS_SEARCH_S, XS_SORT_MATERIAL_ENERGY, legacy stream, no flags. */
 void xs_opts_default(xs_opts *opts);
 
 /* Build a grid on the current CUDA device:

@@ -66,7 +66,7 @@ void xs_opts_default(xs_opts *o)
 {
     if (!o)
         return;
-    o->search = XS_SEARCH_H;
+    o->search = XS_SEARCH_S;
     o->sort = XS_SORT_MATERIAL_ENERGY;
     o->stream = nullptr;
     o->block = 0;

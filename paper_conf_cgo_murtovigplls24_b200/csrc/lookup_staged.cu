@@ -34,20 +34,28 @@ constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the
 #define XS_STAGE_CAP 48
 #endif
 constexpr int kStageCap = XS_STAGE_CAP; // intervals per warp
+#ifndef XS_S_SORT_MIN
+#define XS_S_SORT_MIN 64
+#endif
+constexpr int kSortMinNucs = XS_S_SORT_MIN; // sort a warp's lookups when their material has >= this many nuclides
 constexpr int kIvDoubles = 14;
 struct alignas(16) StageMeta {
     double conc;
     int32_t lo;     // L(q_min) of the nuclide
     int32_t offcnt; // (first staged interval << 16) | intervals, or -1: not staged
 };
-constexpr int kStageWarpBytes =
-    kStageCap * kIvDoubles * 8 + kStageCap * 8 + 32 * (int)sizeof(StageMeta) + ((kStageCap + 15) / 16) * 16;
+constexpr int kStageWarpBytes = kStageCap * kIvDoubles * 8 + kStageCap * 8 + 32 * (int)sizeof(StageMeta) +
+                                32 * 8 + 32 * 4 + ((kStageCap + 15) / 16) * 16;
 
+// The group's per-nuclide state lives in shared memory, not in registers, while the
+// group is computed (registers decide the occupancy of this kernel).
 struct WarpStage {
-    double *rec;     // [kStageCap][kIvDoubles]
-    double *eh;      // [kStageCap] E_hi of each staged interval
-    StageMeta *meta; // [32]
-    uint8_t *owner;  // [kStageCap]
+    double *rec;         // [kStageCap][kIvDoubles]
+    double *eh;          // [kStageCap] E_hi of each staged interval
+    StageMeta *meta;     // [32] conc, lo, staged position
+    const double **pts;  // [32] point row of the nuclide
+    int *cnt;            // [32] intervals of the nuclide's window
+    uint8_t *owner;      // [kStageCap]
 };
 
 __device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
@@ -57,7 +65,9 @@ __device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
     w.rec = reinterpret_cast<double *>(base);
     w.eh = w.rec + kStageCap * kIvDoubles;
     w.meta = reinterpret_cast<StageMeta *>(w.eh + kStageCap);
-    w.owner = reinterpret_cast<uint8_t *>(w.meta + 32);
+    w.pts = reinterpret_cast<const double **>(w.meta + 32);
+    w.cnt = reinterpret_cast<int *>(w.pts + 32);
+    w.owner = reinterpret_cast<uint8_t *>(w.cnt + 32);
     return w;
 }
 
@@ -73,18 +83,27 @@ __device__ __forceinline__ double quotient_markstein(double a, double d, double 
     return __fma_rn(r, y, q0);
 }
 
-// the interpolation of accumulate_pair (reading R8; identical results) from a staged
-// interval record
-__device__ __forceinline__ void accumulate_interval(const double *R, double q, double conc, Acc &A)
+// a staged interval record in registers
+struct IvRec {
+    double2 e, dy, x0, x1, x2, x3, x4;
+};
+
+__device__ __forceinline__ IvRec load_rec(const double *R)
 {
     const double2 *p = reinterpret_cast<const double2 *>(R);
-    const double2 e = p[0], x0 = p[1], x1 = p[2], x2 = p[3], x3 = p[4], x4 = p[5], x5 = p[6];
-    const double f = quotient_markstein(__dsub_rn(e.x, q), e.y, x0.x);
-    A.a0 = __fma_rn(__fma_rn(-f, x1.x, x0.y), conc, A.a0);
-    A.a1 = __fma_rn(__fma_rn(-f, x2.x, x1.y), conc, A.a1);
-    A.a2 = __fma_rn(__fma_rn(-f, x3.x, x2.y), conc, A.a2);
-    A.a3 = __fma_rn(__fma_rn(-f, x4.x, x3.y), conc, A.a3);
-    A.a4 = __fma_rn(__fma_rn(-f, x5.x, x4.y), conc, A.a4);
+    return IvRec{p[0], p[1], p[2], p[3], p[4], p[5], p[6]};
+}
+
+// the interpolation of accumulate_pair (reading R8; identical results) from a staged
+// interval record
+__device__ __forceinline__ void accumulate_interval(const IvRec &v, double q, double conc, Acc &A)
+{
+    const double f = quotient_markstein(__dsub_rn(v.e.x, q), v.dy.x, v.dy.y);
+    A.a0 = __fma_rn(__fma_rn(-f, v.x0.y, v.x0.x), conc, A.a0);
+    A.a1 = __fma_rn(__fma_rn(-f, v.x1.y, v.x1.x), conc, A.a1);
+    A.a2 = __fma_rn(__fma_rn(-f, v.x2.y, v.x2.x), conc, A.a2);
+    A.a3 = __fma_rn(__fma_rn(-f, v.x3.y, v.x3.x), conc, A.a3);
+    A.a4 = __fma_rn(__fma_rn(-f, v.x4.y, v.x4.x), conc, A.a4);
 }
 
 // interval record k of a point row (points k and k+1) into shared memory
@@ -94,14 +113,14 @@ __device__ __forceinline__ void stage_interval(const double *__restrict__ pts, i
     const double2 a0 = __ldg(p), a1 = __ldg(p + 1), a2 = __ldg(p + 2);
     const double2 b0 = __ldg(p + 3), b1 = __ldg(p + 4), b2 = __ldg(p + 5);
     const double d = __dsub_rn(b0.x, a0.x);
-    double2 *o = reinterpret_cast<double2 *>(dst);
-    o[0] = make_double2(b0.x, d);
-    o[1] = make_double2(__drcp_rn(d), b0.y);
-    o[2] = make_double2(__dsub_rn(b0.y, a0.y), b1.x);
-    o[3] = make_double2(__dsub_rn(b1.x, a1.x), b1.y);
-    o[4] = make_double2(__dsub_rn(b1.y, a1.y), b2.x);
-    o[5] = make_double2(__dsub_rn(b2.x, a2.x), b2.y);
-    o[6] = make_double2(__dsub_rn(b2.y, a2.y), 0.0);
+    double2 *o = reinterpret_cast<double2 *>(dst) + 1;
+    o[-1] = make_double2(b0.x, 0.0);
+    o[0] = make_double2(d, __drcp_rn(d));
+    o[1] = make_double2(b0.y, __dsub_rn(b0.y, a0.y));
+    o[2] = make_double2(b1.x, __dsub_rn(b1.x, a1.x));
+    o[3] = make_double2(b1.y, __dsub_rn(b1.y, a1.y));
+    o[4] = make_double2(b2.x, __dsub_rn(b2.x, a2.x));
+    o[5] = make_double2(b2.y, __dsub_rn(b2.y, a2.y));
     *eh = b0.x;
 }
 
@@ -121,6 +140,42 @@ __device__ __forceinline__ int window_count(const double *eh, int cnt, double q)
         }
     }
     return c;
+}
+
+// Bitonic sort of the warp's 2 x 32 (key, value) pairs, ascending over the position
+// e = l * 32 + lane (element l of a lane).  Equal keys keep their own values on both sides
+// of an exchange, so the result is a permutation.
+__device__ __forceinline__ void warp_sort64(uint64_t (&k)[2], uint32_t (&v)[2])
+{
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int size = 2; size <= 64; size <<= 1) {
+#pragma unroll
+        for (int j = size >> 1; j > 0; j >>= 1) {
+            if (j == 32) { // size 64: the partner is this lane's other element
+                if (k[1] < k[0]) {
+                    const uint64_t tk = k[0];
+                    k[0] = k[1];
+                    k[1] = tk;
+                    const uint32_t tv = v[0];
+                    v[0] = v[1];
+                    v[1] = tv;
+                }
+            } else {
+#pragma unroll
+                for (int l = 0; l < 2; l++) {
+                    const int e = l * 32 + lane;
+                    const uint64_t ko = __shfl_xor_sync(0xffffffffu, k[l], j);
+                    const uint32_t vo = __shfl_xor_sync(0xffffffffu, v[l], j);
+                    const bool keep_min = ((e & j) == 0) == ((e & size) == 0);
+                    if (keep_min ? ko < k[l] : ko > k[l]) {
+                        k[l] = ko;
+                        v[l] = vo;
+                    }
+                }
+            }
+        }
+    }
 }
 
 // The lookups in `mine` (one material: row `roww`, nn nuclides; kLpl per lane) accumulate
@@ -149,18 +204,17 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
     for (int g0 = 0; g0 < nn; g0 += 32) {
         // lane t: the window of nuclide g0 + t (H bounds), intervals lo .. lo + cnt - 1
         const int ng = min(32, nn - g0);
-        int lo = 0, cnt = 0;
-        double conc = 0.0;
-        const double *pts = nullptr;
+        __syncwarp(); // the previous group's shared-memory reads are done
         if (lane < ng) {
             const Row rw = load_row(gv, roww + g0 + lane);
-            lo = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_lo, e_lo);
-            cnt = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_hi, e_hi) - lo + 1;
-            conc = rw.conc;
-            pts = rw.pts;
+            const int lo = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_lo, e_lo);
+            ws.cnt[lane] = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_hi, e_hi) - lo + 1;
+            ws.meta[lane] = StageMeta{rw.conc, lo, 0};
+            ws.pts[lane] = rw.pts;
         }
+        __syncwarp();
         for (int b0 = 0; b0 < ng;) { // passes over the group (warp-uniform)
-            const int want = (lane >= b0) ? cnt : 0;
+            const int want = (lane >= b0 && lane < ng) ? ws.cnt[lane] : 0;
             int incl = want;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -171,29 +225,24 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
             const int nfit = __popc(__ballot_sync(0xffffffffu, fits));
             const int T = nfit ? __shfl_sync(0xffffffffu, incl, b0 + nfit - 1) : 0; // intervals staged
             int b1 = b0 + nfit;
-            const int off = incl - want;
             __syncwarp(); // the previous pass's shared-memory reads are done
             if (fits) {
-                ws.meta[lane] = StageMeta{conc, lo, (off << 16) | cnt};
-                for (int k = 0; k < cnt; k++)
+                const int off = incl - want;
+                ws.meta[lane].offcnt = (off << 16) | want;
+                for (int k = 0; k < want; k++)
                     ws.owner[off + k] = (uint8_t)lane;
             }
             if (b1 == b0) { // nuclide b0's window alone exceeds the stage: per-lane H path
                 if (lane == b0)
-                    ws.meta[lane] = StageMeta{conc, lo, -1};
+                    ws.meta[lane].offcnt = -1;
                 b1 = b0 + 1;
             }
             __syncwarp();
             // interval i of the pass is staged by lane i % 32: owner nuclide j, its k-th interval
-            for (int i0 = 0; i0 < T; i0 += 32) {
-                const int i = i0 + lane;
-                const int j = i < T ? ws.owner[i] : b0;
-                const double *pj = reinterpret_cast<const double *>(
-                    __shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(pts), j));
-                const int lo_j = __shfl_sync(0xffffffffu, lo, j);
-                const int off_j = __shfl_sync(0xffffffffu, off, j);
-                if (i < T)
-                    stage_interval(pj, lo_j + (i - off_j), ws.rec + i * kIvDoubles, ws.eh + i);
+            for (int i = lane; i < T; i += 32) {
+                const int j = ws.owner[i];
+                const StageMeta mj = ws.meta[j];
+                stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i);
             }
             __syncwarp();
             for (int jj = b0; jj < b1; jj++) { // ascending nuclide order (R8)
@@ -202,16 +251,29 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
                     const int off_w = m.offcnt >> 16, cnt_w = m.offcnt & 0xFFFF;
                     const double *eh = ws.eh + off_w;
                     const double *R = ws.rec + off_w * kIvDoubles;
-                    if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
+                    if (cnt_w == 1) { // one interval: its record is loaded once for the lane's lookups
+                        const IvRec v = load_rec(R);
+#pragma unroll
+                        for (int l = 0; l < kLpl; l++) {
+                            if (mine[l]) {
+                                accumulate_interval(v, q[l], m.conc, A[l]);
+                                if constexpr (OUTS) {
+                                    if (out_idx)
+                                        out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo;
+                                }
+                            }
+                        }
+                    } else if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
                         const double inf = __longlong_as_double(0x7FF0000000000000ll);
-                        const double e1 = cnt_w > 1 ? eh[0] : inf;
+                        const double e1 = eh[0];
                         const double e2 = cnt_w > 2 ? eh[1] : inf;
                         const double e3 = cnt_w > 3 ? eh[2] : inf;
 #pragma unroll
                         for (int l = 0; l < kLpl; l++) {
                             if (mine[l]) {
+                                // E[lo + k] = eh[k - 1], k = 1..cnt-1
                                 const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
-                                accumulate_interval(R + c * kIvDoubles, q[l], m.conc, A[l]);
+                                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
                                 if constexpr (OUTS) {
                                     if (out_idx)
                                         out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo + c;
@@ -223,7 +285,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
                         for (int l = 0; l < kLpl; l++) {
                             if (mine[l]) {
                                 const int c = window_count(eh, cnt_w, q[l]);
-                                accumulate_interval(R + c * kIvDoubles, q[l], m.conc, A[l]);
+                                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
                                 if constexpr (OUTS) {
                                     if (out_idx)
                                         out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo + c;
@@ -292,8 +354,38 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
                 r[l] = act[l] ? ld_stream(so.slot + j, pol) : 0u;
                 q[l] = act[l] ? ld_stream(so.q_of + r[l], pol) : 0.0;
                 mat[l] = act[l] ? material_of(s_mb, (uint32_t)j) : 0;
-                todo[l] = __ballot_sync(0xffffffffu, act[l]);
             }
+            if constexpr (kLpl == 2) {
+                // one material (the sorted norm): order the warp's 64 lookups by energy, so
+                // each half covers half the energy band and an interval-record load of a
+                // half touches fewer distinct records (shared-memory wavefronts bound S)
+                // (measured: worth its ~600 instructions per 64 lookups only for long nuclide
+                // lists -- large 1.01x, XL 1.05x, small (34 nuclides) 0.89x)
+                const int mat0 = __shfl_sync(0xffffffffu, mat[0], 0);
+                if (__ldg(gv.num_nucs + mat0) >= kSortMinNucs &&
+                    __all_sync(0xffffffffu, (!act[0] || mat[0] == mat0) && (!act[1] || mat[1] == mat0))) {
+                    const int n_act = __popc(__ballot_sync(0xffffffffu, act[0])) +
+                                      __popc(__ballot_sync(0xffffffffu, act[1]));
+                    uint64_t key[2];
+                    uint32_t val[2];
+#pragma unroll
+                    for (int l = 0; l < 2; l++) { // q >= 0: its bits order like its value
+                        key[l] = act[l] ? (uint64_t)__double_as_longlong(q[l]) : ~0ull;
+                        val[l] = r[l];
+                    }
+                    warp_sort64(key, val);
+#pragma unroll
+                    for (int l = 0; l < 2; l++) {
+                        act[l] = l * 32 + lane < n_act;
+                        q[l] = act[l] ? __longlong_as_double((long long)key[l]) : 0.0;
+                        r[l] = val[l];
+                        mat[l] = act[l] ? mat0 : 0;
+                    }
+                }
+            }
+#pragma unroll
+            for (int l = 0; l < kLpl; l++)
+                todo[l] = __ballot_sync(0xffffffffu, act[l]);
             // one round per material among the warp's lookups (sorted: almost always one)
             for (;;) {
                 int src = -1;

@@ -7,7 +7,7 @@ import torch
 from . import _xs
 
 
-def make_opts(search="H", sort="material_energy", stream=None, block=0, energy_bins=0, timing=False,
+def make_opts(search="S", sort="material_energy", stream=None, block=0, energy_bins=0, timing=False,
               split=False, history_len=0):
     o = _xs.xs_opts_default()
     o.search = _xs.SEARCH_NAMES[search] if isinstance(search, str) else int(search)

@@ -278,3 +278,26 @@ def test_xl_hash_sampled(xs, oracle_mod):
     st = g.lookup_range(0, w.lookups, LOOKUP_SEED)  # the bench launch: 125M lookups
     assert st.lookups == w.lookups and w.lookups <= st.hash <= 5 * w.lookups
     g.close()
+
+
+# ------------------------------------------------------------------ large tables, small grids
+@pytest.mark.parametrize("gt", [0, 1, 2])
+@pytest.mark.parametrize("search", ["H", "S"])
+def test_large_tables_small_grid_full(xs, oracle_mod, gt, search):
+    """355 nuclides (fuel 321: S sorts each warp's lookups by energy, long nuclide lists run
+    in several 32-nuclide groups and stage passes) on a 300-point grid, every output of
+    60k lookups against the oracle, with indices"""
+    g = xs.Grid(355, 300, gt, GRID_SEED)
+    P = oracle_mod.Problem(355, 300, gt, GRID_SEED)
+    n = 60_000
+    ref = P.run_range(LOOKUP_SEED, 11, n, idx=True)
+    out, st = g.macro_xs(11, n, LOOKUP_SEED, search=search)
+    assert st.hash == ref["hash"] and st.pairs == ref["pairs"]
+    assert np.array_equal(out.cpu().numpy(), ref["macro"])
+    idx = g.indices(11, n, LOOKUP_SEED, search=search)
+    assert np.array_equal(idx.cpu().numpy(), ref["idx"])
+    for bins in (1, 64):  # wide warp windows: stage passes and the per-lane fallback
+        out, st = g.macro_xs(11, n, LOOKUP_SEED, search=search, energy_bins=bins)
+        assert st.hash == ref["hash"]
+        assert np.array_equal(out.cpu().numpy(), ref["macro"])
+    g.close()

@@ -1,0 +1,7 @@
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_chunks.py -x -q -m gpu -k "S or chunk or ragged or bins or small_full" > gpurun_out/s9_tests.log 2>&1; echo "tests rc=$?" >> gpurun_out/s9_tests.log
+for v in r0s0 r0s1 r1s0 r1s1; do
+  for w in small large; do
+    XS_LIB_VARIANT=$v timeout 300 python bench.py --workload $w --search S --steps 10 --ab '' --no-e2e --no-cpu-baseline > gpurun_out/s9_${v}_${w}.json 2>&1
+  done
+done
