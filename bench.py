@@ -348,6 +348,15 @@ def run_ours(a, w):
         peak_ips = sms * 4 * line["clocks"]["sm_mhz"] * 1e6  # 4 schedulers x 1 warp-instruction/clk
         line["roofline"]["issue"] = {"achieved_warp_inst_per_s": ips, "peak": peak_ips, "frac": ips / peak_ips,
                                      "source": "ncu smsp__inst_executed.sum per launch (profiles/) / live event time"}
+        if rec.get("lsu_wavefronts_per_launch"):
+            # the unit that binds the staged kernel: one L1/shared-memory
+            # data-pipe wavefront per SM per clock
+            wps = rec["lsu_wavefronts_per_launch"] / (mean_lookup_ms / 1e3)
+            peak_wps = sms * line["clocks"]["sm_mhz"] * 1e6
+            line["roofline"]["l1_data_pipe"] = {
+                "achieved_wavefronts_per_s": wps, "peak": peak_wps, "frac": wps / peak_wps,
+                "ncu_pct_of_peak": rec.get("lsu_wavefronts_pct_of_peak"),
+                "source": "ncu shared + global + local LSU wavefronts per launch (profiles/) / live event time"}
     if not a.no_cpu_baseline and R.world == 1:
         cb = cpu_baseline(w, count, a.cpu_seconds)
         # parity of the bench's own configuration on the oracle's sample range

@@ -51,9 +51,17 @@ def main():
                    f"| branch targets uniform % | {num('smsp__sass_average_branch_targets_threads_uniform.pct')} |",
                    f"| FP64 pipe % | {num('sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active')} |",
                    "", "stall samples: " + ", ".join(f"{k} {100*v/tot:.1f}%" for k, v in top), ""]
+            lsu_pct = num("l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed")
+            md.insert(-2, f"L1/shared data pipe (LSU wavefronts) % of peak: {lsu_pct}")
             if "k_lookup" in name:
                 db[key] = {"dram_bytes_per_launch": rd + wr, "warp_inst_per_launch": inst,
-                           "ncu_duration_us": dur_us, "report": os.path.basename(rep), "round": rnd}
+                           "ncu_duration_us": dur_us, "report": os.path.basename(rep), "round": rnd,
+                           "lsu_wavefronts_pct_of_peak": lsu_pct,
+                           "lsu_wavefronts_per_launch": sum(num(k) or 0 for k in (
+                               "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
+                               "l1tex__t_output_wavefronts_pipe_lsu_mem_global_op_ld.sum",
+                               "l1tex__t_output_wavefronts_pipe_lsu_mem_local_op_ld.sum",
+                               "l1tex__t_output_wavefronts_pipe_lsu_mem_local_op_st.sum"))}
         w, s, _ = key.split("/")
         with open(os.path.join(PROF, f"{rnd}_ncu_{w}_{s}.md"), "w") as f:
             f.write("\n".join(md) + "\n")
