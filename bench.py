@@ -264,6 +264,13 @@ def run_ours(a, w):
             "value": R.world * count * a.ab_steps / (ms_max / 1e3),
             "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
         for _ in range(2):
+            step(coarse=True)
+        ms, sts = timed_steps(a.ab_steps, coarse=True)
+        ms_max = driver.max_over_ranks(sum(ms))
+        ab[f"{a.search}/coarse (bucket order without the k_bucket_refine pass)"] = {
+            "value": R.world * count * a.ab_steps / (ms_max / 1e3), "sort_ms": statistics.mean(x.sample_ms for x in sts),
+            "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
+        for _ in range(2):
             step(search="M", sort="none")
         ms, sts = timed_steps(a.ab_steps, search="M", sort="none")
         ms_max = driver.max_over_ranks(sum(ms))

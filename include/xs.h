@@ -97,8 +97,12 @@ enum {
 /* Flags. */
 enum {
     XS_FLAG_TIMING = 1, /* fill the per-phase *_ms fields of xs_stats (CUDA events)          */
-    XS_FLAG_SPLIT = 2   /* sorted modes: the split k_search -> k_interp pair instead of the one
+    XS_FLAG_SPLIT = 2,  /* sorted modes: the split k_search -> k_interp pair instead of the one
                            fused search+interpolation kernel (A/B of the two designs)          */
+    XS_FLAG_COARSE = 4  /* XS_SORT_MATERIAL_ENERGY, fused kernel: stop at the coarse bucket
+                           order (no k_bucket_refine pass; the lookup kernel then gathers each
+                           slot's energy by lookup offset).  A/B of the refine pass; results are
+                           identical either way (any order is a valid ordering)               */
 };
 
 typedef struct xs_opts {

@@ -32,6 +32,7 @@ XS_SEARCH_COUNT = 12
 XS_SORT_NONE, XS_SORT_MATERIAL, XS_SORT_MATERIAL_ENERGY, XS_SORT_HISTORY = 0, 1, 2, 3
 XS_FLAG_TIMING = 1
 XS_FLAG_SPLIT = 2
+XS_FLAG_COARSE = 4
 
 SEARCH_NAMES = {"M": 0, "U1": 1, "U2": 2, "U4": 3, "U8": 4, "B": 5, "M2": 6, "M4": 7, "M8": 8, "W": 9, "H": 10, "S": 11}
 SORT_NAMES = {"none": 0, "material": 1, "material_energy": 2, "history": 3}

@@ -435,6 +435,8 @@ void free_grid(Grid &g)
         cudaFreeHost(g.stats_h);
     cudaFree(g.sq);
     cudaFree(g.si);
+    cudaFree(g.si2);
+    cudaFree(g.jt);
     cudaFree(g.skey);
     cudaFree(g.qs);
     cudaFree(g.Lbuf);

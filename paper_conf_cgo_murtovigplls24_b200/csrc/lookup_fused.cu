@@ -110,7 +110,7 @@ __global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
                 break;
             if (j0 < jend) {
                 r_next = ld_stream(so.slot + j0, pol);
-                q_next = ld_stream(so.q_of + r_next, pol);
+                q_next = so.q ? ld_stream(so.q + j0, pol) : ld_stream(so.q_of + r_next, pol);
             }
         }
     for (int jw = j0 - lane; jw < jend; jw += G) { // warp-uniform trip count
@@ -127,7 +127,7 @@ __global__ void __launch_bounds__(kFusedTpb, ILP2                    ? 3
                 r = r_next;
                 if (j + G < jend) {
                     r_next = ld_stream(so.slot + j + G, pol);
-                    q_next = ld_stream(so.q_of + r_next, pol);
+                    q_next = so.q ? ld_stream(so.q + j + G, pol) : ld_stream(so.q_of + r_next, pol);
                 }
                 mat = material_of(s_mb, (uint32_t)j);
             } else {

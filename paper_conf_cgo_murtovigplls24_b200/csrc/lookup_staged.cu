@@ -352,7 +352,7 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
                 const int j = jw + l * 32 + lane;
                 act[l] = j < jend;
                 r[l] = act[l] ? ld_stream(so.slot + j, pol) : 0u;
-                q[l] = act[l] ? ld_stream(so.q_of + r[l], pol) : 0.0;
+                q[l] = act[l] ? (so.q ? ld_stream(so.q + j, pol) : ld_stream(so.q_of + r[l], pol)) : 0.0;
                 mat[l] = act[l] ? material_of(s_mb, (uint32_t)j) : 0;
             }
             if constexpr (kLpl == 2) {

@@ -1,7 +1,7 @@
 // pipeline.cu -- host orchestration of one xs_lookup_range call.
 //
 //   XS_SORT_NONE                   k_lookup<unsorted>  (sampling fused in)
-//   XS_SORT_MATERIAL[_ENERGY]      bucket sort (4 kernels)  ->  k_lookup<sorted>
+//   XS_SORT_MATERIAL[_ENERGY]      bucket sort (4 kernels, + k_bucket_refine)  ->  k_lookup<sorted>
 //     + XS_FLAG_SPLIT              bucket sort + gather     ->  k_search -> k_interp
 // A range is processed in chunks (slot indices are uint32; scratch stays bounded).  The
 // fused path reads the material bases from device memory (no host round trip); the split
@@ -179,9 +179,11 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         XS_CUDA_TRY(cudaEventRecord(g.ev[1], stream));
         if (sorted) {
             int K = 0;
-            launches += launch_bucket_sort(g, sv, nb, !fused, stream, &K);
-            so.q = g.qs;
-            so.q_of = g.sq;
+            const bool refine = fused && o.sort == XS_SORT_MATERIAL_ENERGY && nb > 1 && !(o.flags & XS_FLAG_COARSE);
+            launches += launch_bucket_sort(g, sv, nb, !fused ? kSortPostGather : (refine ? kSortPostRefine : kSortPostNone),
+                                           stream, &K);
+            so.q = (!fused || refine) ? g.qs : nullptr; // q in slot order when the sort wrote it
+            so.q_of = refine ? nullptr : g.sq;
             so.slot = g.si;
             so.mb_dev = g.base + K;
             so.work = reinterpret_cast<int *>(g.stats_d + 4);

@@ -9,11 +9,15 @@
 //   k_bucket_base    exclusive scan of the bucket totals + material bases (one CTA)
 //   k_bucket_scatter scatter the 4 B lookup offsets to their slots: 68 MB for 17M lookups,
 //                    L2-resident, so the random partial-sector writes merge in L2
-//   k_bucket_gather  (split path only) q in slot order; the fused lookup kernel instead
-//                    prefetches q_of[slot] one grid-stride iteration ahead
+//   k_bucket_refine  (sorted fused path, the default) per group of buckets: a counting sort of
+//                    the bucket's lookups by energy sub-bin (S sub-bins per bucket), writing the
+//                    final slot order and q in slot order (the lookup kernel then streams q
+//                    instead of gathering q_of[slot] at random)
+//   k_bucket_gather  (split path) q in slot order without refining
 // Order inside a bucket is whatever the shared-memory atomics give; results never depend
 // on it (every lookup is independent and the hash is an integer sum).
 #include <algorithm>
+#include <cmath>
 
 #include "lookup_common.cuh"
 
@@ -50,7 +54,8 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, Bucket
             sample_lookup(s, sv, q, mat);
             const int key = bucket_key(s_nb, s_kbase, mat, q);
             atomicAdd(&sh[key], 1u);
-            q_of[j] = q;
+            if (q_of)
+                q_of[j] = q;
             key_of[j] = (uint16_t)key;
             s = lcg_apply(J_tpb, s);
         }
@@ -211,6 +216,184 @@ __global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of,
         q_sorted[j] = __ldg(q_of + __ldg(slot_of + j));
 }
 
+// k_bucket_refine: work group g owns the buckets [g B, g B + B) (under the refine plan every
+// bucket holds ~count/K lookups, so B buckets are ~kRefineTarget lookups), i.e. the slots
+// [base[g B], base[g B + B]); a persistent grid of CTAs takes the groups in turn.  Bucket k
+// of material m covers energies [b / nb[m], (b + 1) / nb[m]) (b = k - kbase[m]); it is cut
+// into S sub-bins, sub = floor((q nb[m] - b) S) clamped to [0, S), and the CTA
+// counting-sorts the group's slots by (bucket, sub-bin): histogram in shared memory, block
+// scan, the refined order assembled in shared memory, then written out coalesced (scattered
+// stores are L2-request bound).  The energy of lookup offset j is recomputed, not gathered:
+// its stream state is J(2 j) s_base with s_base = J(2 first) seed (one Listing-7 jump per
+// chunk, on the host), and J(2 j) is the product of the byte maps J(2 d 256^t), d = byte t
+// of j (tables in shared memory; affine maps of one LCG commute, and arithmetic mod 2^64 maps
+// onto mod 2^63, so this is exactly sample_lookup's state).  A group larger than kRefineCap
+// (a pathological bucket) is handled by re-reading its slots, with scattered stores.  Any
+// order is a valid ordering (results never depend on it): the sub-bin function needs no
+// exact monotonicity, and the order inside a sub-bin is whatever the atomics give.
+constexpr int kRefineTpb = 256;
+constexpr int kRefinePer = 16;                      // slots per thread in registers
+constexpr int kRefineCap = kRefineTpb * kRefinePer; // 4096 slots per group
+constexpr int kRefineBins = 1024;                   // B x S
+constexpr int kRefineTarget = 2560;                 // mean slots per group the plan aims at
+constexpr int kRefineMaxB = 64;
+constexpr int kJumpBytes = 4;                       // lookup offsets < 2^32
+
+__device__ __forceinline__ int refine_bin(double q, double nbm, int b, int kb, int s_log2)
+{
+    const int S = 1 << s_log2;
+    const double x = __dmul_rn(__dsub_rn(__dmul_rn(q, nbm), (double)b), (double)S);
+    int t = (int)x;
+    t = t < 0 ? 0 : (t > S - 1 ? S - 1 : t);
+    return (kb << s_log2) + t;
+}
+
+// energy of lookup offset j (sample_lookup's q): the byte maps applied to the chunk's base
+// state one after the other (nbyte = bytes of the largest offset, uniform)
+__device__ __forceinline__ double energy_of(const Affine *jt, uint64_t s, uint32_t j, int nbyte)
+{
+    for (int t = 0; t < nbyte; t++) {
+        const Affine m = jt[t * 256 + ((j >> (8 * t)) & 255)];
+        s = m.a * s + m.c;
+    }
+    return u63_to_double(lcg_step(s & kMod63));
+}
+
+__global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, int B, int s_log2, int count, int nbyte,
+                                                                  uint64_t s_base, const Affine *__restrict__ jt_g,
+                                                                  const uint32_t *__restrict__ base,
+                                                                  const uint32_t *__restrict__ slot_in,
+                                                                  uint32_t *__restrict__ slot_out,
+                                                                  double *__restrict__ q_out)
+{
+    __shared__ Affine s_jt[kJumpBytes * 256];
+    __shared__ uint32_t s_hist[kRefineBins];
+    __shared__ uint32_t s_bs[kRefineMaxB + 1]; // slot bounds of the group's buckets
+    __shared__ double s_nbm[kRefineMaxB];
+    __shared__ int s_b[kRefineMaxB];
+    __shared__ uint32_t s_wsum[kRefineTpb / 32];
+    extern __shared__ __align__(16) unsigned char s_stage[]; // the refined order: [cap] q, then [cap] offsets
+    double *s_q = reinterpret_cast<double *>(s_stage);
+    uint32_t *s_r = reinterpret_cast<uint32_t *>(s_q + kRefineCap);
+    const int K = bp.K;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    for (int i = tid; i < nbyte * 256; i += kRefineTpb)
+        s_jt[i] = jt_g[i];
+    const int ngroups = (K + B - 1) / B;
+    for (int grp = blockIdx.x; grp < ngroups; grp += gridDim.x) {
+        const int k0 = grp * B, nbk = min(B, K - k0);
+        if (tid <= nbk)
+            s_bs[tid] = (k0 + tid < K) ? __ldg(base + k0 + tid) : (uint32_t)count;
+        if (tid < nbk) {
+            const int k = k0 + tid;
+            int m = 0;
+#pragma unroll
+            for (int mm = 1; mm < kMaterials; mm++)
+                m += (k >= bp.kbase[mm]) ? 1 : 0;
+            s_nbm[tid] = (double)bp.nb[m];
+            s_b[tid] = k - bp.kbase[m];
+        }
+        const int nbins = nbk << s_log2;
+        for (int i = tid; i < nbins; i += kRefineTpb)
+            s_hist[i] = 0u;
+        __syncthreads();
+        const uint32_t s0 = s_bs[0], s1 = s_bs[nbk];
+        const bool regs = s1 - s0 <= (uint32_t)kRefineCap; // CTA-uniform
+        // slots t of a thread increase, so their bucket kb (the last with s_bs[kb] <= t) is
+        // found by walking forward from the previous one
+        int kb = 0;
+        auto bin_of = [&](uint32_t t, double q) {
+            while (kb + 1 < nbk && s_bs[kb + 1] <= t)
+                kb++;
+            return refine_bin(q, s_nbm[kb], s_b[kb], kb, s_log2);
+        };
+        uint32_t r[kRefinePer];
+        double q[kRefinePer];
+        int bin[kRefinePer];
+        if (regs) {
+#pragma unroll
+            for (int u = 0; u < kRefinePer; u++) {
+                const uint32_t t = s0 + tid + u * kRefineTpb;
+                r[u] = t < s1 ? __ldg(slot_in + t) : 0u;
+            }
+#pragma unroll
+            for (int u = 0; u < kRefinePer; u++) {
+                const uint32_t t = s0 + tid + u * kRefineTpb;
+                if (t < s1) {
+                    q[u] = energy_of(s_jt, s_base, r[u], nbyte);
+                    bin[u] = bin_of(t, q[u]);
+                    atomicAdd(&s_hist[bin[u]], 1u);
+                }
+            }
+        } else {
+            for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb)
+                atomicAdd(&s_hist[bin_of(t, energy_of(s_jt, s_base, __ldg(slot_in + t), nbyte))], 1u);
+        }
+        __syncthreads();
+        // exclusive scan of s_hist[0 .. nbins): warp w owns kRows rows of 32 bins (lane =
+        // column: no bank conflicts)
+        constexpr int kRows = kRefineBins / kRefineTpb;
+        const int wb = wid * 32 * kRows;
+        uint32_t wsum = 0;
+#pragma unroll
+        for (int i = 0; i < kRows; i++) {
+            const int k = wb + i * 32 + lane;
+            wsum += k < nbins ? s_hist[k] : 0u;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1)
+            wsum += __shfl_xor_sync(0xffffffffu, wsum, o);
+        if (lane == 0)
+            s_wsum[wid] = wsum;
+        __syncthreads();
+        uint32_t carry = 0;
+        for (int w = 0; w < wid; w++)
+            carry += s_wsum[w];
+#pragma unroll
+        for (int i = 0; i < kRows; i++) {
+            const int k = wb + i * 32 + lane;
+            const uint32_t x = k < nbins ? s_hist[k] : 0u;
+            uint32_t incl = x;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                incl += (lane >= o) ? y : 0u;
+            }
+            if (k < nbins)
+                s_hist[k] = carry + incl - x;
+            carry += __shfl_sync(0xffffffffu, incl, 31);
+        }
+        __syncthreads();
+        if (regs) {
+#pragma unroll
+            for (int u = 0; u < kRefinePer; u++) {
+                const uint32_t t = s0 + tid + u * kRefineTpb;
+                if (t < s1) {
+                    const uint32_t pos = atomicAdd(&s_hist[bin[u]], 1u);
+                    s_r[pos] = r[u];
+                    s_q[pos] = q[u];
+                }
+            }
+            __syncthreads();
+            const uint32_t n = s1 - s0;
+            for (uint32_t i = tid; i < n; i += kRefineTpb) {
+                slot_out[s0 + i] = s_r[i];
+                q_out[s0 + i] = s_q[i];
+            }
+        } else {
+            kb = 0;
+            for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb) {
+                const uint32_t rr = __ldg(slot_in + t);
+                const double qq = energy_of(s_jt, s_base, rr, nbyte);
+                const uint32_t pos = s0 + atomicAdd(&s_hist[bin_of(t, qq)], 1u);
+                slot_out[pos] = rr;
+                q_out[pos] = qq;
+            }
+        }
+        __syncthreads(); // the group's shared state is done before the next group's
+    }
+}
+
 static int sm_count_dev()
 {
     int dev = 0, sms = 0;
@@ -226,15 +409,25 @@ static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
         cudaFree(g.si);
         cudaFree(g.skey);
         cudaFree(g.qs);
+        cudaFree(g.si2);
         g.sq = g.qs = nullptr;
-        g.si = nullptr;
+        g.si = g.si2 = nullptr;
         g.skey = nullptr;
         g.cap = 0;
         XS_CUDA_TRY(cudaMalloc(&g.sq, (size_t)chunk * sizeof(double)));
         XS_CUDA_TRY(cudaMalloc(&g.qs, (size_t)chunk * sizeof(double)));
         XS_CUDA_TRY(cudaMalloc(&g.si, (size_t)chunk * sizeof(uint32_t)));
+        XS_CUDA_TRY(cudaMalloc(&g.si2, (size_t)chunk * sizeof(uint32_t)));
         XS_CUDA_TRY(cudaMalloc(&g.skey, (size_t)chunk * sizeof(uint16_t)));
         g.cap = chunk;
+    }
+    if (!g.jt) { // byte jump tables of k_bucket_refine: jt[t][d] = J(2 d 256^t)
+        static Affine h[kJumpBytes * 256];
+        for (int t = 0; t < kJumpBytes; t++)
+            for (int d = 0; d < 256; d++)
+                h[t * 256 + d] = lcg_jump(2 * (uint64_t)d << (8 * t));
+        XS_CUDA_TRY(cudaMalloc(&g.jt, sizeof(h)));
+        XS_CUDA_TRY(cudaMemcpy(g.jt, h, sizeof(h), cudaMemcpyHostToDevice));
     }
     const int64_t need = (int64_t)ctas * K;
     if (g.hist_cap < need) {
@@ -249,13 +442,13 @@ static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
     }
 }
 
-static BucketPlan make_plan(const Grid &g, int nb_avg)
+static BucketPlan make_plan(const Grid &g, int nb_avg, bool by_lookups)
 {
     BucketPlan bp{};
     double w[kMaterials], W = 0;
     for (int m = 0; m < kMaterials; m++) {
         const double p = (m == 0) ? 1.0 - g.thresholds[11] : g.thresholds[m] - g.thresholds[m - 1];
-        w[m] = p * g.num_nucs[m];
+        w[m] = by_lookups ? p : p * g.num_nucs[m];
         W += w[m];
     }
     // floor(total * share) + at most one bump to 1 per material stays <= 12 * nb_avg
@@ -271,7 +464,7 @@ static BucketPlan make_plan(const Grid &g, int nb_avg)
     return bp;
 }
 
-int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gather, cudaStream_t stream, int *K_out)
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out)
 {
     static bool smem_set[64] = {};
     if (!smem_set[g.device & 63]) {
@@ -281,7 +474,11 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gath
         smem_set[g.device & 63] = true;
     }
     const int64_t cn = sv.count;
-    const BucketPlan bp = make_plan(g, nb_avg);
+    // refine: buckets of equal expected size (the sub-bins give every material its energy
+    // resolution); coarse: cost-weighted, the material that dominates the pairs gets the
+    // finest buckets
+    const bool refine = post == kSortPostRefine && nb_avg > 1;
+    const BucketPlan bp = make_plan(g, nb_avg, refine);
     const int K = bp.K;
     *K_out = K;
     const int sms = sm_count_dev();
@@ -290,12 +487,38 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gath
     ensure_sort_space(g, cn, ctas, K);
     const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
     const size_t smem = (size_t)K * 4;
-    k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, bp, per_cta, J, g.hist, g.sq, g.skey);
+    // refine recomputes energies from lookup offsets: no q_of
+    k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, bp, per_cta, J, g.hist, refine ? nullptr : g.sq, g.skey);
     k_bucket_colscan<<<(K + 31) / 32, 32 * kColWarps, 0, stream>>>(K, ctas, g.hist, g.base);
     k_bucket_base<<<1, 1024, 0, stream>>>(bp, g.base);
-    k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, per_cta, (int)cn, g.hist, g.base, g.skey, g.si);
+    k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, per_cta, (int)cn, g.hist, g.base, g.skey,
+                                                       refine ? g.si2 : g.si);
     XS_CUDA_TRY(cudaGetLastError());
-    if (!with_gather)
+    if (refine) {
+        const double avg = (double)cn / K;
+        const int B = (int)std::max(1.0, std::min<double>(kRefineMaxB, kRefineTarget / std::max(avg, 1.0)));
+        int s_log2 = 0;
+        while ((B << (s_log2 + 1)) <= kRefineBins)
+            s_log2++;
+        int nbyte = 1;
+        while (nbyte < kJumpBytes && (cn - 1) >> (8 * nbyte) > 0)
+            nbyte++;
+        const int rsmem = kRefineCap * 12;
+        if (!g.refine_smem_set) {
+            XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, rsmem));
+            g.refine_smem_set = true;
+        }
+        int per_sm = 0;
+        XS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bucket_refine, kRefineTpb, rsmem));
+        const int ngroups = (K + B - 1) / B;
+        const int rblocks = std::max(1, std::min(ngroups, sms * std::max(per_sm, 1)));
+        k_bucket_refine<<<rblocks, kRefineTpb, rsmem, stream>>>(
+            bp, B, s_log2, (int)cn, nbyte, lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), g.jt, g.base, g.si2,
+            g.si, g.qs);
+        XS_CUDA_TRY(cudaGetLastError());
+        return 5;
+    }
+    if (post != kSortPostGather)
         return 4;
     const int gblocks = (int)std::min<int64_t>((cn + 255) / 256, (int64_t)sms * 8);
     k_bucket_gather<<<gblocks, 256, 0, stream>>>((int)cn, g.si, g.sq, g.qs);

@@ -94,6 +94,9 @@ struct Grid {
     uint32_t *si = nullptr;          // lookup offsets in (material, energy) order  [cap]
     uint16_t *skey = nullptr;        // bucket key by lookup offset                [cap]
     double *qs = nullptr;            // energies in (material, energy) order       [cap]
+    bool refine_smem_set = false;
+    Affine *jt = nullptr;            // refine: byte jump tables J(2 d 256^t), [4][256]
+    uint32_t *si2 = nullptr;         // refine: the coarse slot order before k_bucket_refine [cap]
     int32_t *Lbuf = nullptr;         // split path: lower index of every pair      [lcap]
     int64_t lcap = 0;
     uint32_t *mb_h = nullptr;        // pinned: material bases of the last sort
@@ -184,7 +187,7 @@ SampleView make_sample_view(const Grid &g, uint64_t seed, int64_t first, int64_t
 
 // Lookups of one chunk in (material, energy) order.
 struct SortedView {
-    const double *__restrict__ q;        // split path: energy of sorted slot j (gathered)
+    const double *__restrict__ q;        // energy of sorted slot j (split path, refined sort), else null
     const double *__restrict__ q_of;     // energy by lookup offset
     const uint32_t *__restrict__ slot;   // lookup offset (i - first) of sorted slot j
     const uint32_t *__restrict__ mb_dev; // device copy of matbase (fused path)
@@ -206,10 +209,11 @@ uint64_t grid_checksum(const Grid &g);
 
 // sort.cu: the (material, energy) counting sort of one chunk with `nb_avg` energy buckets
 // per material on average; leaves g.sq (energy by lookup offset) and g.si (slot -> offset)
-// filled and the material bases at g.base + *K_out (device).  with_gather also fills g.qs
-// (energy by slot).  Returns the kernels launched.
-int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, bool with_gather, cudaStream_t stream,
-                       int *K_out);
+// filled and the material bases at g.base + *K_out (device).  Returns the kernels launched.
+// post = kSortPostNone, kSortPostGather (g.qs = q in slot order) or kSortPostRefine
+// (k_bucket_refine: every bucket re-ordered by energy sub-bin, g.si and g.qs rewritten).
+enum { kSortPostNone = 0, kSortPostGather = 1, kSortPostRefine = 2 };
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out);
 
 // lookup_fused.cu: one kernel per lookup batch (search + interpolation in one thread)
 void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, cudaStream_t stream,

@@ -112,6 +112,19 @@ def test_tiny_macro_and_hash(tiny, gt, search, sort, split):
     assert np.array_equal(got, ref["macro"])  # expected bit-exact (R8)
 
 
+@pytest.mark.parametrize("gt", [0, 1, 2])
+@pytest.mark.parametrize("search", ["M", "U2", "W", "H", "S"])
+def test_coarse_order_bitexact(tiny, gt, search):
+    """XS_FLAG_COARSE (no k_bucket_refine pass: coarse buckets, energies gathered by lookup
+    offset) gives the same results as the refined default"""
+    g, P, ref = tiny[gt]
+    out, st = g.macro_xs(0, 100_000, LOOKUP_SEED, search=search, sort="material_energy", coarse=True)
+    assert st.hash == ref["hash"] and st.pairs == ref["pairs"]
+    assert np.array_equal(out.cpu().numpy(), ref["macro"])
+    idx = g.indices(0, 100_000, LOOKUP_SEED, search=search, sort="material_energy", coarse=True)
+    assert np.array_equal(idx.cpu().numpy(), ref["idx"])
+
+
 # ------------------------------------------------------------------ edge cases
 @pytest.mark.parametrize("first,count", [(0, 0), (0, 1), (7, 31), (1000, 257), (99_000, 1000), (3, 4097)])
 @pytest.mark.parametrize("sort,split", PIPES)
