@@ -7,8 +7,9 @@
 //                    offset (coalesced) and histogram the keys in shared memory
 //   k_bucket_colscan per bucket, exclusive scan over CTAs (loads batched by 8)
 //   k_bucket_base    exclusive scan of the bucket totals + material bases (one CTA)
-//   k_bucket_scatter scatter the 4 B lookup offsets to their slots: 68 MB for 17M lookups,
-//                    L2-resident, so the random partial-sector writes merge in L2
+//   k_bucket_scatter scatter the 4 B lookup offsets to their slots, one launch per window of
+//                    buckets whose slots (<= 48 MB) stay L2-resident, so the random
+//                    partial-sector writes merge in L2
 //   k_bucket_refine  (sorted fused path, the default) per group of buckets: a counting sort of
 //                    the bucket's lookups by energy sub-bin (S sub-bins per bucket), writing the
 //                    final slot order and q in slot order (the lookup kernel then streams q
@@ -18,12 +19,14 @@
 // on it (every lookup is independent and the hash is an integer sum).
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 
 #include "lookup_common.cuh"
 
 namespace xs {
 
 constexpr int kSortTpb = 1024;
+constexpr int64_t kScatterWindow = int64_t(48) << 20; // bytes of slots one scatter launch writes
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
                                                             uint32_t *__restrict__ hist, double *__restrict__ q_of,
@@ -179,7 +182,10 @@ __global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, uint32_t *_
     }
 }
 
-__global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int per_cta, int count,
+// Writes the lookups whose key lies in [klo, khi) (one launch per window of buckets: the
+// window's slots, ~kScatterWindow bytes, stay L2-resident while their random partial-sector
+// writes merge; a slot array larger than L2 took DRAM read-modify-writes per 4 B store).
+__global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int khi, int per_cta, int count,
                                                               const uint32_t *__restrict__ hist,
                                                               const uint32_t *__restrict__ base,
                                                               const uint16_t *__restrict__ key_of,
@@ -187,11 +193,12 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int per_cta,
 {
     extern __shared__ uint32_t sh[];
     const uint32_t *h = hist + (int64_t)blockIdx.x * K;
-    for (int k = threadIdx.x; k < K; k += kSortTpb)
+    for (int k = klo + threadIdx.x; k < khi; k += kSortTpb)
         sh[k] = base[k] + h[k];
     __syncthreads();
     const int beg = blockIdx.x * per_cta;
     const int end = min(beg + per_cta, count);
+    const uint32_t span = (uint32_t)(khi - klo);
     // 4 keys in flight per thread, then their shared-memory atomics and 4 B stores
     // (recording each lookup's rank in the count pass to drop the atomics was measured
     // slower)
@@ -203,10 +210,14 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int per_cta,
             kk[u] = key_of[j + u * kSortTpb];
 #pragma unroll
         for (int u = 0; u < 4; u++)
-            slot_of[atomicAdd(&sh[kk[u]], 1u)] = (uint32_t)(j + u * kSortTpb);
+            if (kk[u] - (uint32_t)klo < span)
+                slot_of[atomicAdd(&sh[kk[u]], 1u)] = (uint32_t)(j + u * kSortTpb);
     }
-    for (; j < end; j += kSortTpb)
-        slot_of[atomicAdd(&sh[key_of[j]], 1u)] = (uint32_t)j;
+    for (; j < end; j += kSortTpb) {
+        const uint32_t k = key_of[j];
+        if (k - (uint32_t)klo < span)
+            slot_of[atomicAdd(&sh[k], 1u)] = (uint32_t)j;
+    }
 }
 
 __global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of, const double *__restrict__ q_of,
@@ -249,17 +260,18 @@ __device__ __forceinline__ int refine_bin(double q, double nbm, int b, int kb, i
 }
 
 // energy of lookup offset j (sample_lookup's q): the byte maps applied to the chunk's base
-// state one after the other (nbyte = bytes of the largest offset, uniform)
-__device__ __forceinline__ double energy_of(const Affine *jt, uint64_t s, uint32_t j, int nbyte)
+// state one after the other (an offset byte of 0 maps through the identity)
+__device__ __forceinline__ double energy_of(const Affine *jt, uint64_t s, uint32_t j)
 {
-    for (int t = 0; t < nbyte; t++) {
+#pragma unroll
+    for (int t = 0; t < kJumpBytes; t++) {
         const Affine m = jt[t * 256 + ((j >> (8 * t)) & 255)];
         s = m.a * s + m.c;
     }
     return u63_to_double(lcg_step(s & kMod63));
 }
 
-__global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, int B, int s_log2, int count, int nbyte,
+__global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, int B, int s_log2, int count,
                                                                   uint64_t s_base, const Affine *__restrict__ jt_g,
                                                                   const uint32_t *__restrict__ base,
                                                                   const uint32_t *__restrict__ slot_in,
@@ -267,7 +279,7 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
                                                                   double *__restrict__ q_out)
 {
     __shared__ Affine s_jt[kJumpBytes * 256];
-    __shared__ uint32_t s_hist[kRefineBins];
+    __shared__ uint32_t s_hist[kRefineBins + 1]; // + a dummy bin for the slots past the group
     __shared__ uint32_t s_bs[kRefineMaxB + 1]; // slot bounds of the group's buckets
     __shared__ double s_nbm[kRefineMaxB];
     __shared__ int s_b[kRefineMaxB];
@@ -277,7 +289,7 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
     uint32_t *s_r = reinterpret_cast<uint32_t *>(s_q + kRefineCap);
     const int K = bp.K;
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-    for (int i = tid; i < nbyte * 256; i += kRefineTpb)
+    for (int i = tid; i < kJumpBytes * 256; i += kRefineTpb)
         s_jt[i] = jt_g[i];
     const int ngroups = (K + B - 1) / B;
     for (int grp = blockIdx.x; grp < ngroups; grp += gridDim.x) {
@@ -311,6 +323,8 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
         double q[kRefinePer];
         int bin[kRefinePer];
         if (regs) {
+            // branch-free: positions past the group go to the dummy bin kRefineBins, whose
+            // slots (n, n + 1, ... < kRefineCap) are never written out
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
                 const uint32_t t = s0 + tid + u * kRefineTpb;
@@ -319,15 +333,14 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
                 const uint32_t t = s0 + tid + u * kRefineTpb;
-                if (t < s1) {
-                    q[u] = energy_of(s_jt, s_base, r[u], nbyte);
-                    bin[u] = bin_of(t, q[u]);
-                    atomicAdd(&s_hist[bin[u]], 1u);
-                }
+                q[u] = energy_of(s_jt, s_base, r[u]);
+                const int bb = bin_of(t, q[u]);
+                bin[u] = t < s1 ? bb : kRefineBins;
+                atomicAdd(&s_hist[bin[u]], 1u);
             }
         } else {
             for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb)
-                atomicAdd(&s_hist[bin_of(t, energy_of(s_jt, s_base, __ldg(slot_in + t), nbyte))], 1u);
+                atomicAdd(&s_hist[bin_of(t, energy_of(s_jt, s_base, __ldg(slot_in + t)))], 1u);
         }
         __syncthreads();
         // exclusive scan of s_hist[0 .. nbins): warp w owns kRows rows of 32 bins (lane =
@@ -363,16 +376,15 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
                 s_hist[k] = carry + incl - x;
             carry += __shfl_sync(0xffffffffu, incl, 31);
         }
+        if (tid == 0)
+            s_hist[kRefineBins] = s1 - s0;
         __syncthreads();
         if (regs) {
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
-                const uint32_t t = s0 + tid + u * kRefineTpb;
-                if (t < s1) {
-                    const uint32_t pos = atomicAdd(&s_hist[bin[u]], 1u);
-                    s_r[pos] = r[u];
-                    s_q[pos] = q[u];
-                }
+                const uint32_t pos = atomicAdd(&s_hist[bin[u]], 1u);
+                s_r[pos] = r[u];
+                s_q[pos] = q[u];
             }
             __syncthreads();
             const uint32_t n = s1 - s0;
@@ -384,7 +396,7 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
             kb = 0;
             for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb) {
                 const uint32_t rr = __ldg(slot_in + t);
-                const double qq = energy_of(s_jt, s_base, rr, nbyte);
+                const double qq = energy_of(s_jt, s_base, rr);
                 const uint32_t pos = s0 + atomicAdd(&s_hist[bin_of(t, qq)], 1u);
                 slot_out[pos] = rr;
                 q_out[pos] = qq;
@@ -442,7 +454,7 @@ static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
     }
 }
 
-static BucketPlan make_plan(const Grid &g, int nb_avg, bool by_lookups)
+static BucketPlan make_plan(const Grid &g, int total, bool by_lookups)
 {
     BucketPlan bp{};
     double w[kMaterials], W = 0;
@@ -451,8 +463,7 @@ static BucketPlan make_plan(const Grid &g, int nb_avg, bool by_lookups)
         w[m] = by_lookups ? p : p * g.num_nucs[m];
         W += w[m];
     }
-    // floor(total * share) + at most one bump to 1 per material stays <= 12 * nb_avg
-    const int total = nb_avg > 1 ? kMaterials * (nb_avg - 1) : 0;
+    // floor(total * share) + at most one bump to 1 per material stays <= total + 12
     int k = 0;
     for (int m = 0; m < kMaterials; m++) {
         bp.kbase[m] = k;
@@ -478,7 +489,12 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     // resolution); coarse: cost-weighted, the material that dominates the pairs gets the
     // finest buckets
     const bool refine = post == kSortPostRefine && nb_avg > 1;
-    const BucketPlan bp = make_plan(g, nb_avg, refine);
+    // coarse: 12 (nb_avg - 1) buckets; refine: one bucket per ~kRefineTarget lookups (a
+    // refine group is then one bucket), at most the coarse count
+    const int total_coarse = nb_avg > 1 ? kMaterials * (nb_avg - 1) : 0;
+    const int total = refine ? (int)std::min<int64_t>(total_coarse, std::max<int64_t>(kMaterials, cn / kRefineTarget))
+                             : total_coarse;
+    const BucketPlan bp = make_plan(g, total, refine);
     const int K = bp.K;
     *K_out = K;
     const int sms = sm_count_dev();
@@ -491,8 +507,17 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, bp, per_cta, J, g.hist, refine ? nullptr : g.sq, g.skey);
     k_bucket_colscan<<<(K + 31) / 32, 32 * kColWarps, 0, stream>>>(K, ctas, g.hist, g.base);
     k_bucket_base<<<1, 1024, 0, stream>>>(bp, g.base);
-    k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, per_cta, (int)cn, g.hist, g.base, g.skey,
-                                                       refine ? g.si2 : g.si);
+    // windows of ~equal expected slot counts (refine: equal-size buckets; coarse: cost-weighted
+    // buckets, so the windows are only approximately equal)
+    int64_t win_bytes = kScatterWindow;
+    if (const char *env = std::getenv("XS_SCATTER_WINDOW_MB"))
+        win_bytes = std::max(1ll, std::atoll(env)) << 20;
+    const int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, (cn * 4 + win_bytes - 1) / win_bytes));
+    for (int w = 0; w < nwin; w++) {
+        const int klo = (int)((int64_t)K * w / nwin), khi = (int)((int64_t)K * (w + 1) / nwin);
+        k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, klo, khi, per_cta, (int)cn, g.hist, g.base, g.skey,
+                                                           refine ? g.si2 : g.si);
+    }
     XS_CUDA_TRY(cudaGetLastError());
     if (refine) {
         const double avg = (double)cn / K;
@@ -500,9 +525,6 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
         int s_log2 = 0;
         while ((B << (s_log2 + 1)) <= kRefineBins)
             s_log2++;
-        int nbyte = 1;
-        while (nbyte < kJumpBytes && (cn - 1) >> (8 * nbyte) > 0)
-            nbyte++;
         const int rsmem = kRefineCap * 12;
         if (!g.refine_smem_set) {
             XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, rsmem));
@@ -513,17 +535,17 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
         const int ngroups = (K + B - 1) / B;
         const int rblocks = std::max(1, std::min(ngroups, sms * std::max(per_sm, 1)));
         k_bucket_refine<<<rblocks, kRefineTpb, rsmem, stream>>>(
-            bp, B, s_log2, (int)cn, nbyte, lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), g.jt, g.base, g.si2,
+            bp, B, s_log2, (int)cn, lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), g.jt, g.base, g.si2,
             g.si, g.qs);
         XS_CUDA_TRY(cudaGetLastError());
-        return 5;
+        return 4 + nwin;
     }
     if (post != kSortPostGather)
-        return 4;
+        return 3 + nwin;
     const int gblocks = (int)std::min<int64_t>((cn + 255) / 256, (int64_t)sms * 8);
     k_bucket_gather<<<gblocks, 256, 0, stream>>>((int)cn, g.si, g.sq, g.qs);
     XS_CUDA_TRY(cudaGetLastError());
-    return 5;
+    return 4 + nwin;
 }
 
 } // namespace xs
