@@ -243,35 +243,48 @@ __global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of,
 // order is a valid ordering (results never depend on it): the sub-bin function needs no
 // exact monotonicity, and the order inside a sub-bin is whatever the atomics give.
 constexpr int kRefineTpb = 256;
-constexpr int kRefinePer = 16;                      // slots per thread in registers
-constexpr int kRefineCap = kRefineTpb * kRefinePer; // 4096 slots per group
-constexpr int kRefineBins = 1024;                   // B x S
-constexpr int kRefineTarget = 2560;                 // mean slots per group the plan aims at
+#ifndef XS_REFINE_PER
+#define XS_REFINE_PER 12
+#endif
+#ifndef XS_REFINE_MINB
+#define XS_REFINE_MINB 3
+#endif
+constexpr int kRefinePer = XS_REFINE_PER;           // slots per thread in registers
+constexpr int kRefineCap = kRefineTpb * kRefinePer; // 3072 slots per group
+#ifndef XS_REFINE_BINS
+#define XS_REFINE_BINS 1024
+#endif
+constexpr int kRefineBins = XS_REFINE_BINS;         // B x S
+constexpr int kRefineTarget = kRefineCap * 5 / 8;   // mean slots per group the plan aims at
 constexpr int kRefineMaxB = 64;
 constexpr int kJumpBytes = 4;                       // lookup offsets < 2^32
 
-__device__ __forceinline__ int refine_bin(double q, double nbm, int b, int kb, int s_log2)
+// sub-bin of a lookup from its 63-bit stream state u (q = RN(u) 2^-63): the integer form of
+// floor((q nb - b) S), v = (u >> 20) nb ~ q nb 2^43 (< 2^59); rounding at the bucket edges
+// only moves a lookup into the edge sub-bin (clamped)
+__device__ __forceinline__ int refine_bin(uint64_t u, uint32_t nb, int b, int kb, int s_log2)
 {
+    const uint64_t v = (u >> 20) * (uint64_t)nb;
+    int t = (int)(v >> (43 - s_log2)) - (b << s_log2);
     const int S = 1 << s_log2;
-    const double x = __dmul_rn(__dsub_rn(__dmul_rn(q, nbm), (double)b), (double)S);
-    int t = (int)x;
     t = t < 0 ? 0 : (t > S - 1 ? S - 1 : t);
     return (kb << s_log2) + t;
 }
 
-// energy of lookup offset j (sample_lookup's q): the byte maps applied to the chunk's base
-// state one after the other (an offset byte of 0 maps through the identity)
-__device__ __forceinline__ double energy_of(const Affine *jt, uint64_t s, uint32_t j)
+// stream state of lookup offset j after its energy draw (sample_lookup: q = RN(u) 2^-63): the
+// byte maps applied to the chunk's base state one after the other (an offset byte of 0 maps
+// through the identity)
+__device__ __forceinline__ uint64_t energy_state(const Affine *jt, uint64_t s, uint32_t j)
 {
 #pragma unroll
     for (int t = 0; t < kJumpBytes; t++) {
         const Affine m = jt[t * 256 + ((j >> (8 * t)) & 255)];
         s = m.a * s + m.c;
     }
-    return u63_to_double(lcg_step(s & kMod63));
+    return lcg_step(s & kMod63);
 }
 
-__global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, int B, int s_log2, int count,
+__global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(BucketPlan bp, int B, int s_log2, int count,
                                                                   uint64_t s_base, const Affine *__restrict__ jt_g,
                                                                   const uint32_t *__restrict__ base,
                                                                   const uint32_t *__restrict__ slot_in,
@@ -281,7 +294,7 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
     __shared__ Affine s_jt[kJumpBytes * 256];
     __shared__ uint32_t s_hist[kRefineBins + 1]; // + a dummy bin for the slots past the group
     __shared__ uint32_t s_bs[kRefineMaxB + 1]; // slot bounds of the group's buckets
-    __shared__ double s_nbm[kRefineMaxB];
+    __shared__ uint32_t s_nbm[kRefineMaxB];
     __shared__ int s_b[kRefineMaxB];
     __shared__ uint32_t s_wsum[kRefineTpb / 32];
     extern __shared__ __align__(16) unsigned char s_stage[]; // the refined order: [cap] q, then [cap] offsets
@@ -302,7 +315,7 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
 #pragma unroll
             for (int mm = 1; mm < kMaterials; mm++)
                 m += (k >= bp.kbase[mm]) ? 1 : 0;
-            s_nbm[tid] = (double)bp.nb[m];
+            s_nbm[tid] = (uint32_t)bp.nb[m];
             s_b[tid] = k - bp.kbase[m];
         }
         const int nbins = nbk << s_log2;
@@ -314,10 +327,10 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
         // slots t of a thread increase, so their bucket kb (the last with s_bs[kb] <= t) is
         // found by walking forward from the previous one
         int kb = 0;
-        auto bin_of = [&](uint32_t t, double q) {
+        auto bin_of = [&](uint32_t t, uint64_t u) {
             while (kb + 1 < nbk && s_bs[kb + 1] <= t)
                 kb++;
-            return refine_bin(q, s_nbm[kb], s_b[kb], kb, s_log2);
+            return refine_bin(u, s_nbm[kb], s_b[kb], kb, s_log2);
         };
         uint32_t r[kRefinePer];
         double q[kRefinePer];
@@ -333,19 +346,20 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
                 const uint32_t t = s0 + tid + u * kRefineTpb;
-                q[u] = energy_of(s_jt, s_base, r[u]);
-                const int bb = bin_of(t, q[u]);
+                const uint64_t st = energy_state(s_jt, s_base, r[u]);
+                q[u] = u63_to_double(st);
+                const int bb = bin_of(t, st);
                 bin[u] = t < s1 ? bb : kRefineBins;
                 atomicAdd(&s_hist[bin[u]], 1u);
             }
         } else {
             for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb)
-                atomicAdd(&s_hist[bin_of(t, energy_of(s_jt, s_base, __ldg(slot_in + t)))], 1u);
+                atomicAdd(&s_hist[bin_of(t, energy_state(s_jt, s_base, __ldg(slot_in + t)))], 1u);
         }
         __syncthreads();
         // exclusive scan of s_hist[0 .. nbins): warp w owns kRows rows of 32 bins (lane =
         // column: no bank conflicts)
-        constexpr int kRows = kRefineBins / kRefineTpb;
+        constexpr int kRows = kRefineBins >= kRefineTpb ? kRefineBins / kRefineTpb : 1;
         const int wb = wid * 32 * kRows;
         uint32_t wsum = 0;
 #pragma unroll
@@ -396,8 +410,9 @@ __global__ void __launch_bounds__(kRefineTpb, 3) k_bucket_refine(BucketPlan bp, 
             kb = 0;
             for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb) {
                 const uint32_t rr = __ldg(slot_in + t);
-                const double qq = energy_of(s_jt, s_base, rr);
-                const uint32_t pos = s0 + atomicAdd(&s_hist[bin_of(t, qq)], 1u);
+                const uint64_t st = energy_state(s_jt, s_base, rr);
+                const double qq = u63_to_double(st);
+                const uint32_t pos = s0 + atomicAdd(&s_hist[bin_of(t, st)], 1u);
                 slot_out[pos] = rr;
                 q_out[pos] = qq;
             }
