@@ -178,6 +178,82 @@ __device__ __forceinline__ void warp_sort64(uint64_t (&k)[2], uint32_t (&v)[2])
     }
 }
 
+// One nuclide of a staged group for the lookups in `mine` (ascending nuclide order, R8):
+// the window's interval records are at rec_all + (m.offcnt >> 16) (its upper energies at
+// eh_all + ...); a nuclide whose window was not staged (m.offcnt < 0) takes the per-lane H
+// path.  `col` is the nuclide's column in out_idx.
+template <int GRID, bool OUTS>
+__device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx, int col, const StageMeta m,
+                                                const double *eh_all, const double *rec_all,
+                                                const bool (&mine)[kLpl], const double (&q)[kLpl],
+                                                const uint32_t (&r)[kLpl], int32_t *__restrict__ out_idx,
+                                                Acc (&A)[kLpl])
+{
+    if (m.offcnt >= 0) {
+        const int off_w = m.offcnt >> 16, cnt_w = m.offcnt & 0xFFFF;
+        const double *eh = eh_all + off_w;
+        const double *R = rec_all + off_w * kIvDoubles;
+        if (cnt_w == 1) { // one interval: its record is loaded once for the lane's lookups
+            const IvRec v = load_rec(R);
+#pragma unroll
+            for (int l = 0; l < kLpl; l++) {
+                if (mine[l]) {
+                    accumulate_interval(v, q[l], m.conc, A[l]);
+                    if constexpr (OUTS) {
+                        if (out_idx)
+                            out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo;
+                    }
+                }
+            }
+        } else if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
+            const double inf = __longlong_as_double(0x7FF0000000000000ll);
+            const double e1 = eh[0];
+            const double e2 = cnt_w > 2 ? eh[1] : inf;
+            const double e3 = cnt_w > 3 ? eh[2] : inf;
+#pragma unroll
+            for (int l = 0; l < kLpl; l++) {
+                if (mine[l]) {
+                    // E[lo + k] = eh[k - 1], k = 1..cnt-1
+                    const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
+                    accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
+                    if constexpr (OUTS) {
+                        if (out_idx)
+                            out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
+                    }
+                }
+            }
+        } else {
+#pragma unroll
+            for (int l = 0; l < kLpl; l++) {
+                if (mine[l]) {
+                    const int c = window_count(eh, cnt_w, q[l]);
+                    accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
+                    if constexpr (OUTS) {
+                        if (out_idx)
+                            out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
+                    }
+                }
+            }
+        }
+    } else {
+        const Row rw = load_row(gv, ref_idx);
+#pragma unroll
+        for (int l = 0; l < kLpl; l++) {
+            if (mine[l]) {
+                int e_me = 0;
+                if constexpr (GRID == XS_UNIONIZED)
+                    e_me = union_index<GRID, XS_SEARCH_S>(gv, q[l]);
+                const int L = lower_index<GRID, XS_SEARCH_S>(gv, rw, q[l], e_me);
+                accumulate_pair(rw.pts, L, q[l], rw.conc, A[l]);
+                if constexpr (OUTS) {
+                    if (out_idx)
+                        out_idx[(size_t)r[l] * gv.max_nucs + col] = L;
+                }
+            }
+        }
+    }
+}
+
 // The lookups in `mine` (one material: row `roww`, nn nuclides; kLpl per lane) accumulate
 // every nuclide of the material.  All 32 lanes call it (warp collectives inside).
 template <int GRID, bool OUTS>
@@ -245,74 +321,75 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
                 stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i);
             }
             __syncwarp();
-            for (int jj = b0; jj < b1; jj++) { // ascending nuclide order (R8)
-                const StageMeta m = ws.meta[jj];
-                if (m.offcnt >= 0) {
-                    const int off_w = m.offcnt >> 16, cnt_w = m.offcnt & 0xFFFF;
-                    const double *eh = ws.eh + off_w;
-                    const double *R = ws.rec + off_w * kIvDoubles;
-                    if (cnt_w == 1) { // one interval: its record is loaded once for the lane's lookups
-                        const IvRec v = load_rec(R);
-#pragma unroll
-                        for (int l = 0; l < kLpl; l++) {
-                            if (mine[l]) {
-                                accumulate_interval(v, q[l], m.conc, A[l]);
-                                if constexpr (OUTS) {
-                                    if (out_idx)
-                                        out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo;
-                                }
-                            }
-                        }
-                    } else if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
-                        const double inf = __longlong_as_double(0x7FF0000000000000ll);
-                        const double e1 = eh[0];
-                        const double e2 = cnt_w > 2 ? eh[1] : inf;
-                        const double e3 = cnt_w > 3 ? eh[2] : inf;
-#pragma unroll
-                        for (int l = 0; l < kLpl; l++) {
-                            if (mine[l]) {
-                                // E[lo + k] = eh[k - 1], k = 1..cnt-1
-                                const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
-                                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
-                                if constexpr (OUTS) {
-                                    if (out_idx)
-                                        out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo + c;
-                                }
-                            }
-                        }
-                    } else {
-#pragma unroll
-                        for (int l = 0; l < kLpl; l++) {
-                            if (mine[l]) {
-                                const int c = window_count(eh, cnt_w, q[l]);
-                                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
-                                if constexpr (OUTS) {
-                                    if (out_idx)
-                                        out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = m.lo + c;
-                                }
-                            }
-                        }
-                    }
-                } else {
-                    const Row rw = load_row(gv, roww + g0 + jj);
-#pragma unroll
-                    for (int l = 0; l < kLpl; l++) {
-                        if (mine[l]) {
-                            int e_me = 0;
-                            if constexpr (GRID == XS_UNIONIZED)
-                                e_me = union_index<GRID, XS_SEARCH_S>(gv, q[l]);
-                            const int L = lower_index<GRID, XS_SEARCH_S>(gv, rw, q[l], e_me);
-                            accumulate_pair(rw.pts, L, q[l], rw.conc, A[l]);
-                            if constexpr (OUTS) {
-                                if (out_idx)
-                                    out_idx[(size_t)r[l] * gv.max_nucs + g0 + jj] = L;
-                            }
-                        }
-                    }
-                }
-            }
+            for (int jj = b0; jj < b1; jj++) // ascending nuclide order (R8)
+                compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, ws.meta[jj], ws.eh, ws.rec, mine, q, r,
+                                            out_idx, A);
             b0 = b1;
         }
+    }
+}
+
+// The S path for one warp's kLpl x 32 lookups (act: lane has a lookup; mat per lookup): an
+// optional warp energy sort, then one staged_material round per material among them.
+template <int GRID, bool OUTS>
+__device__ __forceinline__ void warp_lookups(const GridView &gv, const WarpStage &ws, bool (&act)[kLpl],
+                                             double (&q)[kLpl], uint32_t (&r)[kLpl], int (&mat)[kLpl],
+                                             int32_t *__restrict__ out_idx, Acc (&A)[kLpl])
+{
+    const int lane = threadIdx.x & 31;
+    bool mine[kLpl];
+    unsigned todo[kLpl];
+    if constexpr (kLpl == 2) {
+        // one material (the sorted norm): order the warp's 64 lookups by energy, so
+        // each half covers half the energy band and an interval-record load of a
+        // half touches fewer distinct records (shared-memory wavefronts bound S)
+        // (measured: worth its ~600 instructions per 64 lookups only for long nuclide
+        // lists -- large 1.01x, XL 1.05x, small (34 nuclides) 0.89x)
+        const int mat0 = __shfl_sync(0xffffffffu, mat[0], 0);
+        if (__ldg(gv.num_nucs + mat0) >= kSortMinNucs &&
+            __all_sync(0xffffffffu, (!act[0] || mat[0] == mat0) && (!act[1] || mat[1] == mat0))) {
+            const int n_act = __popc(__ballot_sync(0xffffffffu, act[0])) +
+                              __popc(__ballot_sync(0xffffffffu, act[1]));
+            uint64_t key[2];
+            uint32_t val[2];
+#pragma unroll
+            for (int l = 0; l < 2; l++) { // q >= 0: its bits order like its value
+                key[l] = act[l] ? (uint64_t)__double_as_longlong(q[l]) : ~0ull;
+                val[l] = r[l];
+            }
+            warp_sort64(key, val);
+#pragma unroll
+            for (int l = 0; l < 2; l++) {
+                act[l] = l * 32 + lane < n_act;
+                q[l] = act[l] ? __longlong_as_double((long long)key[l]) : 0.0;
+                r[l] = val[l];
+                mat[l] = act[l] ? mat0 : 0;
+            }
+        }
+    }
+#pragma unroll
+    for (int l = 0; l < kLpl; l++)
+        todo[l] = __ballot_sync(0xffffffffu, act[l]);
+    // one round per material among the warp's lookups (sorted: almost always one)
+    for (;;) {
+        int src = -1;
+#pragma unroll
+        for (int l = kLpl - 1; l >= 0; l--)
+            src = todo[l] ? l * 32 + __ffs(todo[l]) - 1 : src;
+        if (src < 0)
+            break;
+        int mw = mat[0];
+#pragma unroll
+        for (int l = 1; l < kLpl; l++)
+            mw = (src >> 5) == l ? mat[l] : mw;
+        const int mat_w = __shfl_sync(0xffffffffu, mw, src & 31);
+#pragma unroll
+        for (int l = 0; l < kLpl; l++) {
+            mine[l] = act[l] && mat[l] == mat_w;
+            todo[l] &= ~__ballot_sync(0xffffffffu, mine[l]);
+        }
+        staged_material<GRID, OUTS>(gv, mat_w * gv.max_nucs, __ldg(gv.num_nucs + mat_w), mine, q, r, ws,
+                                    out_idx, A);
     }
 }
 
@@ -341,12 +418,11 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
             break;
         const int jend = min(count, c * kStChunk + kStChunk);
         for (int jw = c * kStChunk; jw < jend; jw += 32 * kLpl) {
-            bool act[kLpl], mine[kLpl];
+            bool act[kLpl];
             double q[kLpl];
             uint32_t r[kLpl];
             int mat[kLpl];
             Acc A[kLpl];
-            unsigned todo[kLpl];
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
                 const int j = jw + l * 32 + lane;
@@ -355,58 +431,7 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
                 q[l] = act[l] ? (so.q ? ld_stream(so.q + j, pol) : ld_stream(so.q_of + r[l], pol)) : 0.0;
                 mat[l] = act[l] ? material_of(s_mb, (uint32_t)j) : 0;
             }
-            if constexpr (kLpl == 2) {
-                // one material (the sorted norm): order the warp's 64 lookups by energy, so
-                // each half covers half the energy band and an interval-record load of a
-                // half touches fewer distinct records (shared-memory wavefronts bound S)
-                // (measured: worth its ~600 instructions per 64 lookups only for long nuclide
-                // lists -- large 1.01x, XL 1.05x, small (34 nuclides) 0.89x)
-                const int mat0 = __shfl_sync(0xffffffffu, mat[0], 0);
-                if (__ldg(gv.num_nucs + mat0) >= kSortMinNucs &&
-                    __all_sync(0xffffffffu, (!act[0] || mat[0] == mat0) && (!act[1] || mat[1] == mat0))) {
-                    const int n_act = __popc(__ballot_sync(0xffffffffu, act[0])) +
-                                      __popc(__ballot_sync(0xffffffffu, act[1]));
-                    uint64_t key[2];
-                    uint32_t val[2];
-#pragma unroll
-                    for (int l = 0; l < 2; l++) { // q >= 0: its bits order like its value
-                        key[l] = act[l] ? (uint64_t)__double_as_longlong(q[l]) : ~0ull;
-                        val[l] = r[l];
-                    }
-                    warp_sort64(key, val);
-#pragma unroll
-                    for (int l = 0; l < 2; l++) {
-                        act[l] = l * 32 + lane < n_act;
-                        q[l] = act[l] ? __longlong_as_double((long long)key[l]) : 0.0;
-                        r[l] = val[l];
-                        mat[l] = act[l] ? mat0 : 0;
-                    }
-                }
-            }
-#pragma unroll
-            for (int l = 0; l < kLpl; l++)
-                todo[l] = __ballot_sync(0xffffffffu, act[l]);
-            // one round per material among the warp's lookups (sorted: almost always one)
-            for (;;) {
-                int src = -1;
-#pragma unroll
-                for (int l = kLpl - 1; l >= 0; l--)
-                    src = todo[l] ? l * 32 + __ffs(todo[l]) - 1 : src;
-                if (src < 0)
-                    break;
-                int mw = mat[0];
-#pragma unroll
-                for (int l = 1; l < kLpl; l++)
-                    mw = (src >> 5) == l ? mat[l] : mw;
-                const int mat_w = __shfl_sync(0xffffffffu, mw, src & 31);
-#pragma unroll
-                for (int l = 0; l < kLpl; l++) {
-                    mine[l] = act[l] && mat[l] == mat_w;
-                    todo[l] &= ~__ballot_sync(0xffffffffu, mine[l]);
-                }
-                staged_material<GRID, OUTS>(gv, mat_w * gv.max_nucs, __ldg(gv.num_nucs + mat_w), mine, q, r, ws,
-                                            out_idx, A);
-            }
+            warp_lookups<GRID, OUTS>(gv, ws, act, q, r, mat, out_idx, A);
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
                 if (act[l]) {
