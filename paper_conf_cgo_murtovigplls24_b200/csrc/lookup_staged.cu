@@ -21,6 +21,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_LPL
 #define XS_S_LPL 2
 #endif
+#ifndef XS_S_PF
+#define XS_S_PF 1
+#endif
 constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the staged windows
 
 // ---- XS_SEARCH_S: staged warp windows -----------------------------------
@@ -193,16 +196,17 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
         const int off_w = m.offcnt >> 16, cnt_w = m.offcnt & 0xFFFF;
         const double *eh = eh_all + off_w;
         const double *R = rec_all + off_w * kIvDoubles;
+        // branch-free over the lane's lookups, so their FP64 chains interleave: a lookup
+        // that is not `mine` accumulates with concentration +0, fma(micro, +0, acc) == acc
+        // exactly (micro is finite and acc is never -0)
         if (cnt_w == 1) { // one interval: its record is loaded once for the lane's lookups
             const IvRec v = load_rec(R);
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
-                if (mine[l]) {
-                    accumulate_interval(v, q[l], m.conc, A[l]);
-                    if constexpr (OUTS) {
-                        if (out_idx)
-                            out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo;
-                    }
+                accumulate_interval(v, q[l], mine[l] ? m.conc : 0.0, A[l]);
+                if constexpr (OUTS) {
+                    if (out_idx && mine[l])
+                        out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo;
                 }
             }
         } else if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
@@ -212,14 +216,12 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             const double e3 = cnt_w > 3 ? eh[2] : inf;
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
-                if (mine[l]) {
-                    // E[lo + k] = eh[k - 1], k = 1..cnt-1
-                    const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
-                    accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
-                    if constexpr (OUTS) {
-                        if (out_idx)
-                            out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
-                    }
+                // E[lo + k] = eh[k - 1], k = 1..cnt-1
+                const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
+                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], mine[l] ? m.conc : 0.0, A[l]);
+                if constexpr (OUTS) {
+                    if (out_idx && mine[l])
+                        out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
                 }
             }
         } else {
@@ -416,6 +418,19 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
         c = __shfl_sync(0xffffffffu, c, 0);
         if (c * kStChunk >= count)
             break;
+#if XS_S_PF
+        // chunks are handed out in order: the chunk one resident wave ahead is fetched by some
+        // warp about one chunk-time from now -- bring its slots and energies into L2
+        if (so.q) {
+            const int cp = c + (int)(gridDim.x * (kStTpb / 32));
+            constexpr int kQLines = kStChunk * 8 / 128, kSLines = kStChunk * 4 / 128;
+            if (lane < kQLines + kSLines && cp * kStChunk < count) {
+                const void *a = lane < kQLines ? (const void *)(so.q + (size_t)cp * kStChunk + lane * 16)
+                                               : (const void *)(so.slot + (size_t)cp * kStChunk + (lane - kQLines) * 32);
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+            }
+        }
+#endif
         const int jend = min(count, c * kStChunk + kStChunk);
         for (int jw = c * kStChunk; jw < jend; jw += 32 * kLpl) {
             bool act[kLpl];
