@@ -12,17 +12,20 @@ namespace xs {
 
 constexpr int kStTpb = 256;
 #ifndef XS_S_MIN_BLOCKS
-#define XS_S_MIN_BLOCKS 3
+#define XS_S_MIN_BLOCKS 2
 #endif
 #ifndef XS_S_CHUNK
-#define XS_S_CHUNK 128
+#define XS_S_CHUNK 256
 #endif
 constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pulls one at a time)
 #ifndef XS_S_LPL
-#define XS_S_LPL 2
+#define XS_S_LPL 4
 #endif
 #ifndef XS_S_PF
 #define XS_S_PF 1
+#endif
+#ifndef XS_S_WSORT
+#define XS_S_WSORT 0
 #endif
 constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the staged windows
 
@@ -145,28 +148,37 @@ __device__ __forceinline__ int window_count(const double *eh, int cnt, double q)
     return c;
 }
 
-// Bitonic sort of the warp's 2 x 32 (key, value) pairs, ascending over the position
-// e = l * 32 + lane (element l of a lane).  Equal keys keep their own values on both sides
-// of an exchange, so the result is a permutation.
-__device__ __forceinline__ void warp_sort64(uint64_t (&k)[2], uint32_t (&v)[2])
+// Bitonic sort of the warp's kLpl x 32 (key, value) pairs (kLpl a power of two), ascending
+// over the position e = l * 32 + lane (element l of a lane).  Equal keys keep their own
+// values on both sides of an exchange, so the result is a permutation.
+__device__ __forceinline__ void warp_sort(uint64_t (&k)[kLpl], uint32_t (&v)[kLpl])
 {
+    static_assert((kLpl & (kLpl - 1)) == 0, "warp_sort needs a power-of-two kLpl");
     const int lane = threadIdx.x & 31;
 #pragma unroll
-    for (int size = 2; size <= 64; size <<= 1) {
+    for (int size = 2; size <= 32 * kLpl; size <<= 1) {
 #pragma unroll
         for (int j = size >> 1; j > 0; j >>= 1) {
-            if (j == 32) { // size 64: the partner is this lane's other element
-                if (k[1] < k[0]) {
-                    const uint64_t tk = k[0];
-                    k[0] = k[1];
-                    k[1] = tk;
-                    const uint32_t tv = v[0];
-                    v[0] = v[1];
-                    v[1] = tv;
+            if (j >= 32) { // the partner is element l ^ (j / 32) of this lane
+                const int jl = j >> 5;
+#pragma unroll
+                for (int l = 0; l < kLpl; l++) {
+                    if ((l & jl) == 0) {
+                        const int l2 = l | jl;
+                        const bool asc = ((l * 32) & size) == 0;
+                        if (asc ? k[l2] < k[l] : k[l2] > k[l]) {
+                            const uint64_t tk = k[l];
+                            k[l] = k[l2];
+                            k[l2] = tk;
+                            const uint32_t tv = v[l];
+                            v[l] = v[l2];
+                            v[l2] = tv;
+                        }
+                    }
                 }
             } else {
 #pragma unroll
-                for (int l = 0; l < 2; l++) {
+                for (int l = 0; l < kLpl; l++) {
                     const int e = l * 32 + lane;
                     const uint64_t ko = __shfl_xor_sync(0xffffffffu, k[l], j);
                     const uint32_t vo = __shfl_xor_sync(0xffffffffu, v[l], j);
@@ -341,27 +353,31 @@ __device__ __forceinline__ void warp_lookups(const GridView &gv, const WarpStage
     const int lane = threadIdx.x & 31;
     bool mine[kLpl];
     unsigned todo[kLpl];
-    if constexpr (kLpl == 2) {
-        // one material (the sorted norm): order the warp's 64 lookups by energy, so
-        // each half covers half the energy band and an interval-record load of a
-        // half touches fewer distinct records (shared-memory wavefronts bound S)
-        // (measured: worth its ~600 instructions per 64 lookups only for long nuclide
-        // lists -- large 1.01x, XL 1.05x, small (34 nuclides) 0.89x)
+#if XS_S_WSORT
+    {
+        // one material (the sorted norm): order the warp's lookups by energy, so each
+        // element l covers a slice of the energy band and an interval-record load touches
+        // fewer distinct records (shared-memory wavefronts bound S)
         const int mat0 = __shfl_sync(0xffffffffu, mat[0], 0);
-        if (__ldg(gv.num_nucs + mat0) >= kSortMinNucs &&
-            __all_sync(0xffffffffu, (!act[0] || mat[0] == mat0) && (!act[1] || mat[1] == mat0))) {
-            const int n_act = __popc(__ballot_sync(0xffffffffu, act[0])) +
-                              __popc(__ballot_sync(0xffffffffu, act[1]));
-            uint64_t key[2];
-            uint32_t val[2];
+        bool same = true;
 #pragma unroll
-            for (int l = 0; l < 2; l++) { // q >= 0: its bits order like its value
+        for (int l = 0; l < kLpl; l++)
+            same = same && (!act[l] || mat[l] == mat0);
+        if (__ldg(gv.num_nucs + mat0) >= kSortMinNucs && __all_sync(0xffffffffu, same)) {
+            int n_act = 0;
+#pragma unroll
+            for (int l = 0; l < kLpl; l++)
+                n_act += __popc(__ballot_sync(0xffffffffu, act[l]));
+            uint64_t key[kLpl];
+            uint32_t val[kLpl];
+#pragma unroll
+            for (int l = 0; l < kLpl; l++) { // q >= 0: its bits order like its value
                 key[l] = act[l] ? (uint64_t)__double_as_longlong(q[l]) : ~0ull;
                 val[l] = r[l];
             }
-            warp_sort64(key, val);
+            warp_sort(key, val);
 #pragma unroll
-            for (int l = 0; l < 2; l++) {
+            for (int l = 0; l < kLpl; l++) {
                 act[l] = l * 32 + lane < n_act;
                 q[l] = act[l] ? __longlong_as_double((long long)key[l]) : 0.0;
                 r[l] = val[l];
@@ -369,6 +385,7 @@ __device__ __forceinline__ void warp_lookups(const GridView &gv, const WarpStage
             }
         }
     }
+#endif
 #pragma unroll
     for (int l = 0; l < kLpl; l++)
         todo[l] = __ballot_sync(0xffffffffu, act[l]);
