@@ -27,6 +27,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_WSORT
 #define XS_S_WSORT 0
 #endif
+#ifndef XS_S_ALL
+#define XS_S_ALL 1
+#endif
 constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the staged windows
 
 // ---- XS_SEARCH_S: staged warp windows -----------------------------------
@@ -197,7 +200,7 @@ __device__ __forceinline__ void warp_sort(uint64_t (&k)[kLpl], uint32_t (&v)[kLp
 // the window's interval records are at rec_all + (m.offcnt >> 16) (its upper energies at
 // eh_all + ...); a nuclide whose window was not staged (m.offcnt < 0) takes the per-lane H
 // path.  `col` is the nuclide's column in out_idx.
-template <int GRID, bool OUTS>
+template <int GRID, bool OUTS, bool ALL = false>
 __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx, int col, const StageMeta m,
                                                 const double *eh_all, const double *rec_all,
                                                 const bool (&mine)[kLpl], const double (&q)[kLpl],
@@ -215,7 +218,7 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             const IvRec v = load_rec(R);
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
-                accumulate_interval(v, q[l], mine[l] ? m.conc : 0.0, A[l]);
+                accumulate_interval(v, q[l], (ALL || mine[l]) ? m.conc : 0.0, A[l]);
                 if constexpr (OUTS) {
                     if (out_idx && mine[l])
                         out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo;
@@ -230,7 +233,7 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             for (int l = 0; l < kLpl; l++) {
                 // E[lo + k] = eh[k - 1], k = 1..cnt-1
                 const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
-                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], mine[l] ? m.conc : 0.0, A[l]);
+                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], (ALL || mine[l]) ? m.conc : 0.0, A[l]);
                 if constexpr (OUTS) {
                     if (out_idx && mine[l])
                         out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
@@ -286,6 +289,13 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
         mx = mine[l] ? fmax(mx, q[l]) : mx;
     }
     const double q_lo = warp_min(mn), q_hi = warp_max(mx);
+#if XS_S_ALL
+    bool mine_all = true;
+#pragma unroll
+    for (int l = 0; l < kLpl; l++)
+        mine_all = mine_all && mine[l];
+    const bool all_mine = __all_sync(0xffffffffu, mine_all);
+#endif
     int e_lo = 0, e_hi = 0;
     if constexpr (GRID == XS_UNIONIZED) {
         e_lo = union_index<GRID, XS_SEARCH_S>(gv, q_lo);
@@ -335,9 +345,16 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
                 stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i);
             }
             __syncwarp();
-            for (int jj = b0; jj < b1; jj++) // ascending nuclide order (R8)
-                compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, ws.meta[jj], ws.eh, ws.rec, mine, q, r,
-                                            out_idx, A);
+#if XS_S_ALL
+            if (all_mine) // every lookup of the warp is this material's (the sorted norm): no selects
+                for (int jj = b0; jj < b1; jj++) // ascending nuclide order (R8)
+                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ws.meta[jj], ws.eh, ws.rec, mine, q,
+                                                      r, out_idx, A);
+            else
+#endif
+                for (int jj = b0; jj < b1; jj++) // ascending nuclide order (R8)
+                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, ws.meta[jj], ws.eh, ws.rec, mine, q, r,
+                                                out_idx, A);
             b0 = b1;
         }
     }

@@ -251,9 +251,6 @@ constexpr int kRefineTpb = 256;
 #endif
 constexpr int kRefinePer = XS_REFINE_PER;           // slots per thread in registers
 constexpr int kRefineCap = kRefineTpb * kRefinePer; // 3072 slots per group
-#ifndef XS_REFINE_MATCH
-#define XS_REFINE_MATCH 0
-#endif
 #ifndef XS_REFINE_BINS
 #define XS_REFINE_BINS 1024
 #endif
@@ -296,12 +293,6 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
 {
     __shared__ Affine s_jt[kJumpBytes * 256];
     __shared__ uint32_t s_hist[kRefineBins + 1]; // + a dummy bin for the slots past the group
-#if XS_REFINE_MATCH
-    // per-warp counters [warp][bin] (u16: a group holds <= kRefineCap slots): ranks come from
-    // warp matches and plain read-modify-writes by one leader lane per distinct bin -- no
-    // shared-memory atomics (2 cycles per lane with a return value)
-    __shared__ uint16_t s_wcnt[kRefineTpb / 32][kRefineBins + 2];
-#endif
     __shared__ uint32_t s_bs[kRefineMaxB + 1]; // slot bounds of the group's buckets
     __shared__ uint32_t s_nbm[kRefineMaxB];
     __shared__ int s_b[kRefineMaxB];
@@ -314,7 +305,6 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
     for (int i = tid; i < kJumpBytes * 256; i += kRefineTpb)
         s_jt[i] = jt_g[i];
     const int ngroups = (K + B - 1) / B;
-    constexpr bool regs_possible = true;
     for (int grp = blockIdx.x; grp < ngroups; grp += gridDim.x) {
         const int k0 = grp * B, nbk = min(B, K - k0);
         if (tid <= nbk)
@@ -329,13 +319,6 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
             s_b[tid] = k - bp.kbase[m];
         }
         const int nbins = nbk << s_log2;
-#if XS_REFINE_MATCH
-        if (regs_possible) {
-            for (int i = lane; i <= kRefineBins; i += 32)
-                s_wcnt[wid][i] = 0;
-            __syncwarp();
-        }
-#endif
         for (int i = tid; i < nbins; i += kRefineTpb)
             s_hist[i] = 0u;
         __syncthreads();
@@ -367,35 +350,13 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
                 q[u] = u63_to_double(st);
                 const int bb = bin_of(t, st);
                 bin[u] = t < s1 ? bb : kRefineBins;
-#if XS_REFINE_MATCH
-                const unsigned peers = __match_any_sync(0xffffffffu, bin[u]);
-                if (lane == __ffs(peers) - 1)
-                    s_wcnt[wid][bin[u]] += (uint16_t)__popc(peers);
-                __syncwarp();
-#else
                 atomicAdd(&s_hist[bin[u]], 1u);
-#endif
             }
         } else {
             for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb)
                 atomicAdd(&s_hist[bin_of(t, energy_state(s_jt, s_base, __ldg(slot_in + t)))], 1u);
         }
         __syncthreads();
-#if XS_REFINE_MATCH
-        if (regs) { // bin totals, and each warp's offset inside every bin
-            for (int b2 = tid; b2 < nbins; b2 += kRefineTpb) {
-                uint32_t run = 0;
-#pragma unroll
-                for (int w = 0; w < kRefineTpb / 32; w++) {
-                    const uint32_t x = s_wcnt[w][b2];
-                    s_wcnt[w][b2] = (uint16_t)run;
-                    run += x;
-                }
-                s_hist[b2] = run;
-            }
-            __syncthreads();
-        }
-#endif
         // exclusive scan of s_hist[0 .. nbins): warp w owns kRows rows of 32 bins (lane =
         // column: no bank conflicts)
         constexpr int kRows = kRefineBins >= kRefineTpb ? kRefineBins / kRefineTpb : 1;
@@ -435,19 +396,7 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
         if (regs) {
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
-#if XS_REFINE_MATCH
-                // bin start + this warp's offset in the bin + rank among the warp's peers
-                const unsigned peers = __match_any_sync(0xffffffffu, bin[u]);
-                const int lead = __ffs(peers) - 1;
-                const uint32_t wo = s_wcnt[wid][bin[u]];
-                const uint32_t pos = s_hist[bin[u]] + wo + __popc(peers & ((1u << lane) - 1u));
-                __syncwarp();
-                if (lane == lead)
-                    s_wcnt[wid][bin[u]] = (uint16_t)(wo + __popc(peers));
-                __syncwarp();
-#else
                 const uint32_t pos = atomicAdd(&s_hist[bin[u]], 1u);
-#endif
                 if (pos < (uint32_t)kRefineCap) {
                     s_r[pos] = r[u];
                     s_q[pos] = q[u];
