@@ -472,13 +472,17 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
             uint32_t r[kLpl];
             int mat[kLpl];
             Acc A[kLpl];
+            // material of the iteration's slots: one (warp-uniform) lookup when they all lie
+            // in one material's run of slots (the sorted norm), else per lookup
+            const int mw = material_of(s_mb, (uint32_t)jw);
+            const bool one_mat = (uint32_t)min(jend, jw + 32 * kLpl) <= s_mb[mw + 1];
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
                 const int j = jw + l * 32 + lane;
                 act[l] = j < jend;
                 r[l] = act[l] ? ld_stream(so.slot + j, pol) : 0u;
                 q[l] = act[l] ? (so.q ? ld_stream(so.q + j, pol) : ld_stream(so.q_of + r[l], pol)) : 0.0;
-                mat[l] = act[l] ? material_of(s_mb, (uint32_t)j) : 0;
+                mat[l] = !act[l] ? 0 : (one_mat ? mw : material_of(s_mb, (uint32_t)j));
             }
             warp_lookups<GRID, OUTS>(gv, ws, act, q, r, mat, out_idx, A);
 #pragma unroll
