@@ -364,6 +364,20 @@ def run_ours(a, w):
                 "achieved_wavefronts_per_s": wps, "peak": peak_wps, "frac": wps / peak_wps,
                 "ncu_pct_of_peak": rec.get("lsu_wavefronts_pct_of_peak"),
                 "source": "ncu shared + global + local LSU wavefronts per launch (profiles/) / live event time"}
+    try:  # SURVEY.md §8d's measured random-gather roofline (tools/l2_gather.cu on this pool's B200)
+        with open(os.path.join(ROOT, "profiles", "l2_gather.json")) as f:
+            lg = json.load(f)
+        key = {"small": "small_points_37MB", "large": "large_points_193MB", "large-U": "large_points_193MB",
+               "XL": "xl_points_4.07GB"}.get(w.name)
+        if key and lg["gathers"].get(key):
+            gp = lg["gathers"][key]["GBps_useful"]
+            line["roofline"]["random_gather"] = {
+                "peak": gp, "unit": "GB/s", "frac": achieved / gp, "buffer": key,
+                "source": "profiles/l2_gather.json: random 96 B record gathers over a buffer the size of this "
+                          "workload's point records (L2-resident for small); frac > 1 = the sort turns the "
+                          "random gather into shared accesses"}
+    except Exception:
+        pass
     if not a.no_cpu_baseline and R.world == 1:
         cb = cpu_baseline(w, count, a.cpu_seconds)
         # parity of the bench's own configuration on the oracle's sample range
