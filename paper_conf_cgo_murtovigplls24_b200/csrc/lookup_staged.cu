@@ -516,12 +516,8 @@ void launch_staged(int grid_type, int blocks, int tpb, cudaStream_t stream, cons
                                              : pick_staged<XS_HASH>(outs);
     (void)tpb; // one configuration: 256 threads, XS_S_MIN_BLOCKS CTAs per SM
     const int smem = (kStTpb / 32) * kStageWarpBytes;
-    XS_CUDA_TRY(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    int per_sm = 0;
-    XS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, kStTpb, smem));
-    int dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int per_sm = resident_ctas((const void *)f, kStTpb, smem);
+    const int sms = sm_count_cached();
     const int want = (int)((sv.count + kStTpb - 1) / kStTpb);
     const int nb = std::max(1, std::min(want, sms * std::max(per_sm, 1)));
     (void)blocks;

@@ -8,6 +8,8 @@
 // path brings them back (52 B) to size the pair buffer exactly.
 #include <algorithm>
 #include <cstdlib>
+#include <mutex>
+#include <vector>
 
 #include "lookup_common.cuh"
 
@@ -57,12 +59,45 @@ template <int GRID> static SearchPtsFn pick_pts(int search)
 }
 
 // ---- helpers ---------------------------------------------------------------------------------
-static int sm_count()
+int sm_count_cached()
 {
-    int dev = 0, sms = 0;
+    static int cache[64] = {};
+    int dev = 0;
     cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    return sms > 0 ? sms : 148;
+    int &c = cache[dev & 63];
+    if (!c) {
+        int sms = 0;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        c = sms > 0 ? sms : 148;
+    }
+    return c;
+}
+
+static int sm_count() { return sm_count_cached(); }
+
+int resident_ctas(const void *f, int tpb, int smem)
+{
+    struct Entry {
+        const void *f;
+        int dev, tpb, smem, per_sm;
+    };
+    static std::mutex mu;
+    static std::vector<Entry> cache;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lock(mu);
+    for (const Entry &e : cache)
+        if (e.f == f && e.dev == dev && e.tpb == tpb && e.smem == smem)
+            return e.per_sm;
+    XS_CUDA_TRY(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+#ifdef XS_MAX_CARVEOUT
+    XS_CUDA_TRY(cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
+#endif
+    int per_sm = 0;
+    XS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, f, tpb, smem));
+    per_sm = std::max(per_sm, 1);
+    cache.push_back(Entry{f, dev, tpb, smem, per_sm});
+    return per_sm;
 }
 
 static bool is_device_accessible(const void *p)
@@ -236,7 +271,11 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             copied_pending[buf] = true;
         }
         XS_CUDA_TRY(cudaEventRecord(g.ev[5], stream));
-        if (timing) {
+        // timing: a chunk's events are read before the next chunk reuses them; the last
+        // chunk's (device-only) times are read after the call's final synchronisation, so
+        // timing adds no host round trip inside the last chunk
+        const bool last = c0 + chunk >= count;
+        if (timing && !(last && !host_out)) {
             XS_CUDA_TRY(cudaStreamSynchronize(stream));
             float a = 0, b = 0, c = 0, d = 0;
             cudaEventElapsedTime(&a, g.ev[1], g.ev[2]);
@@ -262,6 +301,15 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
     XS_CUDA_TRY(cudaStreamSynchronize(stream));
     float total = 0;
     XS_CUDA_TRY(cudaEventElapsedTime(&total, g.ev[0], g.ev[6]));
+    if (timing && !host_out && count > 0) { // the last chunk's phases (deferred above)
+        float a = 0, b = 0, c = 0;
+        cudaEventElapsedTime(&a, g.ev[1], g.ev[2]);
+        cudaEventElapsedTime(&b, g.ev[2], g.ev[4]);
+        cudaEventElapsedTime(&c, g.ev[2], g.ev[3]);
+        sample_ms += a;
+        lookup_ms += b;
+        search_ms += c;
+    }
     if (st) {
         st->hash = g.stats_h[0];
         st->pairs = g.stats_h[1];

@@ -423,13 +423,7 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
     }
 }
 
-static int sm_count_dev()
-{
-    int dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    return sms > 0 ? sms : 148;
-}
+static int sm_count_dev() { return sm_count_cached(); }
 
 static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
 {
@@ -494,12 +488,10 @@ static BucketPlan make_plan(const Grid &g, int total, bool by_lookups)
 
 int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out)
 {
-    static bool smem_set[64] = {};
-    if (!smem_set[g.device & 63]) {
-        const int bytes = kMaterials * kMaxEnergyBins * 4;
-        XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_count, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
-        XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
-        smem_set[g.device & 63] = true;
+    {
+        const int bytes = kMaterials * kMaxEnergyBins * 4; // the largest histogram a plan can ask for
+        resident_ctas((const void *)k_bucket_count, kSortTpb, bytes);
+        resident_ctas((const void *)k_bucket_scatter, kSortTpb, bytes);
     }
     const int64_t cn = sv.count;
     // refine: buckets of equal expected size (the sub-bins give every material its energy
@@ -543,12 +535,7 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
         while ((B << (s_log2 + 1)) <= kRefineBins)
             s_log2++;
         const int rsmem = kRefineCap * 12;
-        if (!g.refine_smem_set) {
-            XS_CUDA_TRY(cudaFuncSetAttribute(k_bucket_refine, cudaFuncAttributeMaxDynamicSharedMemorySize, rsmem));
-            g.refine_smem_set = true;
-        }
-        int per_sm = 0;
-        XS_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bucket_refine, kRefineTpb, rsmem));
+        const int per_sm = resident_ctas((const void *)k_bucket_refine, kRefineTpb, rsmem);
         const int ngroups = (K + B - 1) / B;
         const int rblocks = std::max(1, std::min(ngroups, sms * std::max(per_sm, 1)));
         k_bucket_refine<<<rblocks, kRefineTpb, rsmem, stream>>>(

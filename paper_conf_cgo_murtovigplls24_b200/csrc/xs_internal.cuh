@@ -94,7 +94,6 @@ struct Grid {
     uint32_t *si = nullptr;          // lookup offsets in (material, energy) order  [cap]
     uint16_t *skey = nullptr;        // bucket key by lookup offset                [cap]
     double *qs = nullptr;            // energies in (material, energy) order       [cap]
-    bool refine_smem_set = false;
     Affine *jt = nullptr;            // refine: byte jump tables J(2 d 256^t), [4][256]
     uint32_t *si2 = nullptr;         // refine: the coarse slot order before k_bucket_refine [cap]
     int32_t *Lbuf = nullptr;         // split path: lower index of every pair      [lcap]
@@ -239,6 +238,15 @@ constexpr int kSearchTpb = 256;
 constexpr int kInterpTpb = 256;
 
 // pipeline.cu
+// Resident CTAs per SM of kernel f at (tpb threads, smem bytes of dynamic shared memory) on
+// the current device; the first call per (device, f, smem) also raises f's dynamic-shared-
+// memory limit to smem.  Cached, so a call costs no driver round trip after the first (the
+// attribute and occupancy queries used to run on every launch).  A maximum shared-memory
+// carveout for every kernel (-DXS_MAX_CARVEOUT) measured 1% slower: the lookup kernel's
+// global loads lose L1.
+int resident_ctas(const void *f, int tpb, int smem);
+int sm_count_cached();
+
 void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
                  int32_t *out_idx, xs_stats *st);
 void run_bezier_surface(int ni, int nj, int64_t res_i, int64_t res_j, int dtype, int variant, const void *P,
