@@ -37,7 +37,8 @@ constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the
 // in a compact array (the window count reads them), 32 window descriptors and the owner
 // lane of every staged interval.  Interval record (112 B = 7 x 16 B): the quantities of
 // reading R8 that do not depend on q, rounded exactly as accumulate_pair rounds them,
-//   [0] E_hi  [1] d = E_hi - E_lo  [2] y = RN(1/d)  [3 + 2c] X_c,hi  [4 + 2c] dX_c = X_c,hi - X_c,lo
+//   [0] E_hi  [1] conc of the nuclide  [2] d = E_hi - E_lo  [3] y = RN(1/d)
+//   [4 + 2c] X_c,hi  [5 + 2c] dX_c = X_c,hi - X_c,lo
 // so a pair costs one subtraction, Markstein's quotient (3 ops) and 10 FMAs.
 #ifndef XS_STAGE_CAP
 #define XS_STAGE_CAP 48
@@ -116,14 +117,15 @@ __device__ __forceinline__ void accumulate_interval(const IvRec &v, double q, do
 }
 
 // interval record k of a point row (points k and k+1) into shared memory
-__device__ __forceinline__ void stage_interval(const double *__restrict__ pts, int k, double *dst, double *eh)
+__device__ __forceinline__ void stage_interval(const double *__restrict__ pts, int k, double *dst, double *eh,
+                                               double conc)
 {
     const double2 *p = reinterpret_cast<const double2 *>(pts) + (size_t)(uint32_t)k * 3;
     const double2 a0 = __ldg(p), a1 = __ldg(p + 1), a2 = __ldg(p + 2);
     const double2 b0 = __ldg(p + 3), b1 = __ldg(p + 4), b2 = __ldg(p + 5);
     const double d = __dsub_rn(b0.x, a0.x);
     double2 *o = reinterpret_cast<double2 *>(dst) + 1;
-    o[-1] = make_double2(b0.x, 0.0);
+    o[-1] = make_double2(b0.x, conc); // the nuclide's concentration rides in the pad slot
     o[0] = make_double2(d, __drcp_rn(d));
     o[1] = make_double2(b0.y, __dsub_rn(b0.y, a0.y));
     o[2] = make_double2(b1.x, __dsub_rn(b1.x, a1.x));
@@ -201,14 +203,14 @@ __device__ __forceinline__ void warp_sort(uint64_t (&k)[kLpl], uint32_t (&v)[kLp
 // eh_all + ...); a nuclide whose window was not staged (m.offcnt < 0) takes the per-lane H
 // path.  `col` is the nuclide's column in out_idx.
 template <int GRID, bool OUTS, bool ALL = false>
-__device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx, int col, const StageMeta m,
-                                                const double *eh_all, const double *rec_all,
+__device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx, int col, const int offcnt,
+                                                const StageMeta *mp, const double *eh_all, const double *rec_all,
                                                 const bool (&mine)[kLpl], const double (&q)[kLpl],
                                                 const uint32_t (&r)[kLpl], int32_t *__restrict__ out_idx,
                                                 Acc (&A)[kLpl])
 {
-    if (m.offcnt >= 0) {
-        const int off_w = m.offcnt >> 16, cnt_w = m.offcnt & 0xFFFF;
+    if (offcnt >= 0) {
+        const int off_w = offcnt >> 16, cnt_w = offcnt & 0xFFFF;
         const double *eh = eh_all + off_w;
         const double *R = rec_all + off_w * kIvDoubles;
         // branch-free over the lane's lookups, so their FP64 chains interleave: a lookup
@@ -218,10 +220,10 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             const IvRec v = load_rec(R);
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
-                accumulate_interval(v, q[l], (ALL || mine[l]) ? m.conc : 0.0, A[l]);
+                accumulate_interval(v, q[l], (ALL || mine[l]) ? v.e.y : 0.0, A[l]);
                 if constexpr (OUTS) {
                     if (out_idx && mine[l])
-                        out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo;
+                        out_idx[(size_t)r[l] * gv.max_nucs + col] = mp->lo;
                 }
             }
         } else if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
@@ -233,10 +235,11 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             for (int l = 0; l < kLpl; l++) {
                 // E[lo + k] = eh[k - 1], k = 1..cnt-1
                 const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
-                accumulate_interval(load_rec(R + c * kIvDoubles), q[l], (ALL || mine[l]) ? m.conc : 0.0, A[l]);
+                const IvRec v = load_rec(R + c * kIvDoubles);
+                accumulate_interval(v, q[l], (ALL || mine[l]) ? v.e.y : 0.0, A[l]);
                 if constexpr (OUTS) {
                     if (out_idx && mine[l])
-                        out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
+                        out_idx[(size_t)r[l] * gv.max_nucs + col] = mp->lo + c;
                 }
             }
         } else {
@@ -244,10 +247,11 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             for (int l = 0; l < kLpl; l++) {
                 if (mine[l]) {
                     const int c = window_count(eh, cnt_w, q[l]);
-                    accumulate_interval(load_rec(R + c * kIvDoubles), q[l], m.conc, A[l]);
+                    const IvRec v = load_rec(R + c * kIvDoubles);
+                    accumulate_interval(v, q[l], v.e.y, A[l]);
                     if constexpr (OUTS) {
                         if (out_idx)
-                            out_idx[(size_t)r[l] * gv.max_nucs + col] = m.lo + c;
+                            out_idx[(size_t)r[l] * gv.max_nucs + col] = mp->lo + c;
                     }
                 }
             }
@@ -342,19 +346,28 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
             for (int i = lane; i < T; i += 32) {
                 const int j = ws.owner[i];
                 const StageMeta mj = ws.meta[j];
-                stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i);
+                stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i, mj.conc);
             }
             __syncwarp();
+            // ascending nuclide order (R8); the next nuclide's window descriptor is read one
+            // nuclide ahead (the record load depends on it)
+            int oc = ws.meta[b0].offcnt;
 #if XS_S_ALL
-            if (all_mine) // every lookup of the warp is this material's (the sorted norm): no selects
-                for (int jj = b0; jj < b1; jj++) // ascending nuclide order (R8)
-                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ws.meta[jj], ws.eh, ws.rec, mine, q,
-                                                      r, out_idx, A);
-            else
+            if (all_mine) { // every lookup of the warp is this material's (the sorted norm): no selects
+                for (int jj = b0; jj < b1; jj++) {
+                    const int oc_next = jj + 1 < b1 ? ws.meta[jj + 1].offcnt : 0;
+                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.eh, ws.rec,
+                                                      mine, q, r, out_idx, A);
+                    oc = oc_next;
+                }
+            } else
 #endif
-                for (int jj = b0; jj < b1; jj++) // ascending nuclide order (R8)
-                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, ws.meta[jj], ws.eh, ws.rec, mine, q, r,
-                                                out_idx, A);
+                for (int jj = b0; jj < b1; jj++) {
+                    const int oc_next = jj + 1 < b1 ? ws.meta[jj + 1].offcnt : 0;
+                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.eh, ws.rec, mine, q,
+                                                r, out_idx, A);
+                    oc = oc_next;
+                }
             b0 = b1;
         }
     }
