@@ -524,7 +524,9 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     int64_t win_bytes = std::min<int64_t>(kScatterWindow, std::max<int64_t>(int64_t(16) << 20, cn * 4 / 8));
     if (const char *env = std::getenv("XS_SCATTER_WINDOW_MB"))
         win_bytes = std::max(1ll, std::atoll(env)) << 20;
-    const int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, (cn * 4 + win_bytes - 1) / win_bytes));
+    int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, (cn * 4 + win_bytes - 1) / win_bytes));
+    if (const char *env = std::getenv("XS_TEST_SCATTER_WINDOWS")) // test hook: force the window count
+        nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, std::atoll(env)));
     for (int w = 0; w < nwin; w++) {
         const int klo = (int)((int64_t)K * w / nwin), khi = (int)((int64_t)K * (w + 1) / nwin);
         k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, klo, khi, per_cta, (int)cn, g.hist, g.base, g.skey,

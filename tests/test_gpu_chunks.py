@@ -43,3 +43,35 @@ def test_many_chunks_match_oracle(chunk):
     env = dict(os.environ, XS_TEST_MAX_CHUNK=str(chunk))
     r = subprocess.run([sys.executable, "-c", SCRIPT], capture_output=True, text=True, env=env, timeout=900)
     assert r.returncode == 0 and "CHUNKS OK" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
+
+
+WINDOW_SCRIPT = r"""
+import sys; sys.path.insert(0, %r)
+import numpy as np
+import oracle
+import paper_conf_cgo_murtovigplls24_b200 as xs
+for gt in (0, 1, 2):
+    P = oracle.Problem(68, 1000, gt, 42)
+    ref = P.run_range(1070, 5, 100_000, idx=True)
+    with xs.Grid(68, 1000, gt, 42) as g:
+        for search in ("H", "S"):
+            for coarse in (False, True):
+                out, st = g.macro_xs(5, 100_000, 1070, search=search, coarse=coarse)
+                assert st.hash == ref["hash"] and st.pairs == ref["pairs"], (gt, search, coarse)
+                assert np.array_equal(out.cpu().numpy(), ref["macro"]), (gt, search, coarse)
+                idx = g.indices(5, 100_000, 1070, search=search, coarse=coarse)
+                assert np.array_equal(idx.cpu().numpy(), ref["idx"]), (gt, search, coarse)
+print("WINDOWS OK")
+""" % ROOT
+
+
+@pytest.mark.parametrize("windows", [2, 7, 39])
+def test_scatter_windows_match_oracle(windows):
+    """the windowed scatter (one launch per window of buckets) with the window count forced
+    (XS_TEST_SCATTER_WINDOWS): every bucket is written by exactly one window"""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    env = dict(os.environ, XS_TEST_SCATTER_WINDOWS=str(windows))
+    r = subprocess.run([sys.executable, "-c", WINDOW_SCRIPT], capture_output=True, text=True, env=env, timeout=900)
+    assert r.returncode == 0 and "WINDOWS OK" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
