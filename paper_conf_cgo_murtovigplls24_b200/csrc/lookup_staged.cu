@@ -447,6 +447,7 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
     k_lookup_staged(GridView gv, SortedView so, int count, double *__restrict__ out_, int32_t *__restrict__ out_idx_,
                     unsigned long long *__restrict__ stats)
 {
+    pdl_wait(); // the sort's outputs (and the work counter it zeroed) are complete
     double *__restrict__ out = OUTS ? out_ : nullptr;
     int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
     extern __shared__ __align__(16) unsigned char st_smem[];
@@ -534,7 +535,7 @@ void launch_staged(int grid_type, int blocks, int tpb, cudaStream_t stream, cons
     const int want = (int)((sv.count + kStTpb - 1) / kStTpb);
     const int nb = std::max(1, std::min(want, sms * std::max(per_sm, 1)));
     (void)blocks;
-    f<<<nb, kStTpb, smem, stream>>>(gv, so, (int)sv.count, out, out_idx, stats);
+    launch_pdl(f, nb, kStTpb, smem, stream, gv, so, (int)sv.count, out, out_idx, stats);
     XS_CUDA_TRY(cudaGetLastError());
 }
 

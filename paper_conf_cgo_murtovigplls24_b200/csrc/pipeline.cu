@@ -221,8 +221,7 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             so.q_of = refine ? nullptr : g.sq;
             so.slot = g.si;
             so.mb_dev = g.base + K;
-            so.work = reinterpret_cast<int *>(g.stats_d + 4);
-            XS_CUDA_TRY(cudaMemsetAsync(so.work, 0, sizeof(int), stream));
+            so.work = reinterpret_cast<int *>(g.stats_d + 4); // zeroed by k_bucket_count
             if (!fused) {
                 XS_CUDA_TRY(cudaMemcpyAsync(g.mb_h, g.base + K, (kMaterials + 1) * sizeof(uint32_t),
                                             cudaMemcpyDeviceToHost, stream));

@@ -30,8 +30,12 @@ constexpr int64_t kScatterWindow = int64_t(48) << 20; // max bytes of slots one 
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
                                                             uint32_t *__restrict__ hist, double *__restrict__ q_of,
-                                                            uint16_t *__restrict__ key_of)
+                                                            uint16_t *__restrict__ key_of, int *__restrict__ work)
 {
+    pdl_wait();
+    pdl_trigger();
+    if (work && blockIdx.x == 0 && threadIdx.x == 0)
+        *work = 0; // the lookup kernel's work-queue counter (read only after this kernel)
     extern __shared__ uint32_t sh[];
     __shared__ int s_nb[kMaterials], s_kbase[kMaterials];
     const int K = bp.K;
@@ -78,6 +82,8 @@ constexpr int kColWarps = 8;
 __global__ void __launch_bounds__(32 * kColWarps) k_bucket_colscan(int K, int ctas, uint32_t *hist,
                                                                     uint32_t *__restrict__ total)
 {
+    pdl_wait();
+    pdl_trigger();
     __shared__ uint32_t part[kColWarps][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int k = blockIdx.x * 32 + lane;
@@ -133,6 +139,8 @@ __global__ void __launch_bounds__(32 * kColWarps) k_bucket_colscan(int K, int ct
 // base[K + m] = first slot of material m, base[K + 12] = count.
 __global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, uint32_t *__restrict__ base)
 {
+    pdl_wait();
+    pdl_trigger();
     __shared__ uint32_t wsum[32];
     const int K = bp.K;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -191,6 +199,8 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int
                                                               const uint16_t *__restrict__ key_of,
                                                               uint32_t *__restrict__ slot_of)
 {
+    pdl_wait();
+    pdl_trigger();
     extern __shared__ uint32_t sh[];
     const uint32_t *h = hist + (int64_t)blockIdx.x * K;
     for (int k = klo + threadIdx.x; k < khi; k += kSortTpb)
@@ -291,6 +301,8 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
                                                                   uint32_t *__restrict__ slot_out,
                                                                   double *__restrict__ q_out)
 {
+    pdl_wait();
+    pdl_trigger();
     __shared__ Affine s_jt[kJumpBytes * 256];
     __shared__ uint32_t s_hist[kRefineBins + 1]; // + a dummy bin for the slots past the group
     __shared__ uint32_t s_bs[kRefineMaxB + 1]; // slot bounds of the group's buckets
@@ -513,9 +525,10 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
     const size_t smem = (size_t)K * 4;
     // refine recomputes energies from lookup offsets: no q_of
-    k_bucket_count<<<ctas, kSortTpb, smem, stream>>>(sv, bp, per_cta, J, g.hist, refine ? nullptr : g.sq, g.skey);
-    k_bucket_colscan<<<(K + 31) / 32, 32 * kColWarps, 0, stream>>>(K, ctas, g.hist, g.base);
-    k_bucket_base<<<1, 1024, 0, stream>>>(bp, g.base);
+    launch_pdl(k_bucket_count, ctas, kSortTpb, (int)smem, stream, sv, bp, per_cta, J, g.hist,
+               refine ? nullptr : g.sq, g.skey, reinterpret_cast<int *>(g.stats_d + 4));
+    launch_pdl(k_bucket_colscan, (K + 31) / 32, 32 * kColWarps, 0, stream, K, ctas, g.hist, g.base);
+    launch_pdl(k_bucket_base, 1, 1024, 0, stream, bp, g.base);
     // windows of ~equal expected slot counts (refine: equal-size buckets; coarse: cost-weighted
     // buckets, so the windows are only approximately equal)
     // window: 1/8 of the slot array, within [16, 48] MB -- more windows keep each one's
@@ -529,8 +542,8 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
         nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, std::atoll(env)));
     for (int w = 0; w < nwin; w++) {
         const int klo = (int)((int64_t)K * w / nwin), khi = (int)((int64_t)K * (w + 1) / nwin);
-        k_bucket_scatter<<<ctas, kSortTpb, smem, stream>>>(K, klo, khi, per_cta, (int)cn, g.hist, g.base, g.skey,
-                                                           refine ? g.si2 : g.si);
+        launch_pdl(k_bucket_scatter, ctas, kSortTpb, (int)smem, stream, K, klo, khi, per_cta, (int)cn, g.hist, g.base,
+                   g.skey, refine ? g.si2 : g.si);
     }
     XS_CUDA_TRY(cudaGetLastError());
     if (refine) {
@@ -543,9 +556,9 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
         const int per_sm = resident_ctas((const void *)k_bucket_refine, kRefineTpb, rsmem);
         const int ngroups = (K + B - 1) / B;
         const int rblocks = std::max(1, std::min(ngroups, sms * std::max(per_sm, 1)));
-        k_bucket_refine<<<rblocks, kRefineTpb, rsmem, stream>>>(
-            bp, B, s_log2, (int)cn, lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), g.jt, g.base, g.si2,
-            g.si, g.qs);
+        launch_pdl(k_bucket_refine, rblocks, kRefineTpb, rsmem, stream, bp, B, s_log2, (int)cn,
+                   lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), (const Affine *)g.jt,
+                   (const uint32_t *)g.base, (const uint32_t *)g.si2, g.si, g.qs);
         XS_CUDA_TRY(cudaGetLastError());
         return 4 + nwin;
     }

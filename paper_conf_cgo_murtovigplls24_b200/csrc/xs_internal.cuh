@@ -245,6 +245,43 @@ constexpr int kInterpTpb = 256;
 // carveout for every kernel (-DXS_MAX_CARVEOUT) measured 1% slower: the lookup kernel's
 // global loads lose L1.
 int resident_ctas(const void *f, int tpb, int smem);
+
+// Programmatic dependent launch (PDL) between the kernels of one lookup step: a kernel is
+// launched with programmatic stream serialisation, so its CTAs can be scheduled while its
+// predecessor drains; every such kernel starts with pdl_wait() (griddepcontrol.wait: blocks
+// until the predecessor grid has completed and its memory is visible -- before any read of
+// its outputs) and then pdl_trigger() (lets its own successor start launching).  Without
+// the launch attribute both are no-ops.  XS_PDL=0 turns it off.
+#ifndef XS_PDL
+#define XS_PDL 1
+#endif
+__device__ __forceinline__ void pdl_wait()
+{
+#if XS_PDL
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
+}
+__device__ __forceinline__ void pdl_trigger()
+{
+#if XS_PDL
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
+}
+template <typename... KArgs, typename... Args>
+inline void launch_pdl(void (*kernel)(KArgs...), int grid, int block, int smem, cudaStream_t stream, Args... args)
+{
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = XS_PDL ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    XS_CUDA_TRY(cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...));
+}
 int sm_count_cached();
 
 void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
