@@ -511,6 +511,17 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
         }
     }
     reduce_stats<kStTpb>(my_hash, my_pairs, stats);
+    if (so.pub && threadIdx.x == 0) { // the last CTA publishes the totals to host-mapped memory
+        __threadfence();
+        if (atomicAdd(so.done, 1u) == gridDim.x - 1) {
+            __threadfence();
+            const unsigned long long h = atomicAdd(stats + 0, 0ull), pr = atomicAdd(stats + 1, 0ull);
+            volatile unsigned long long *p = so.pub;
+            p[0] = h;
+            p[1] = pr;
+            __threadfence_system();
+        }
+    }
 }
 
 using StagedFn = void (*)(GridView, SortedView, int, double *, int32_t *, unsigned long long *);

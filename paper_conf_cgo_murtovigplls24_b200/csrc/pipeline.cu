@@ -191,6 +191,7 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         }
     }
     bool copied_pending[2] = {false, false};
+    bool published = false; // the last S chunk wrote the stats to the (mapped) pinned mirror
     const int64_t stage_half = std::min(count, chunk) * 5;
     if (!g.mb_h)
         XS_CUDA_TRY(cudaMallocHost(&g.mb_h, 32 * sizeof(uint32_t)));
@@ -222,6 +223,11 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
             so.slot = g.si;
             so.mb_dev = g.base + K;
             so.work = reinterpret_cast<int *>(g.stats_d + 4); // zeroed by k_bucket_count
+            if (fused && o.search == XS_SEARCH_S && c0 + chunk >= count) { // the last chunk of S
+                so.done = reinterpret_cast<unsigned int *>(g.stats_d + 5);   // publishes the stats
+                so.pub = reinterpret_cast<unsigned long long *>(g.stats_h);
+                published = true;
+            }
             if (!fused) {
                 XS_CUDA_TRY(cudaMemcpyAsync(g.mb_h, g.base + K, (kMaterials + 1) * sizeof(uint32_t),
                                             cudaMemcpyDeviceToHost, stream));
@@ -295,7 +301,8 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
     for (int b = 0; b < 2; b++) // the call's stream covers every outstanding copy
         if (copied_pending[b])
             XS_CUDA_TRY(cudaStreamWaitEvent(stream, g.ev_copied[b], 0));
-    XS_CUDA_TRY(cudaMemcpyAsync(g.stats_h, g.stats_d, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, stream));
+    if (!published || count == 0)
+        XS_CUDA_TRY(cudaMemcpyAsync(g.stats_h, g.stats_d, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, stream));
     XS_CUDA_TRY(cudaEventRecord(g.ev[6], stream));
     XS_CUDA_TRY(cudaStreamSynchronize(stream));
     float total = 0;

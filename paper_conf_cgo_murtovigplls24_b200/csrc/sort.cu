@@ -30,12 +30,15 @@ constexpr int64_t kScatterWindow = int64_t(48) << 20; // max bytes of slots one 
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
                                                             uint32_t *__restrict__ hist, double *__restrict__ q_of,
-                                                            uint16_t *__restrict__ key_of, int *__restrict__ work)
+                                                            uint16_t *__restrict__ key_of,
+                                                            unsigned long long *__restrict__ ctl)
 {
     pdl_wait();
     pdl_trigger();
-    if (work && blockIdx.x == 0 && threadIdx.x == 0)
-        *work = 0; // the lookup kernel's work-queue counter (read only after this kernel)
+    if (ctl && blockIdx.x == 0 && threadIdx.x == 0) { // the lookup kernel's work-queue counter
+        ctl[0] = 0;                                 // and CTA-completion count (read only
+        ctl[1] = 0;                                 // after this kernel)
+    }
     extern __shared__ uint32_t sh[];
     __shared__ int s_nb[kMaterials], s_kbase[kMaterials];
     const int K = bp.K;
@@ -526,7 +529,7 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     const size_t smem = (size_t)K * 4;
     // refine recomputes energies from lookup offsets: no q_of
     launch_pdl(k_bucket_count, ctas, kSortTpb, (int)smem, stream, sv, bp, per_cta, J, g.hist,
-               refine ? nullptr : g.sq, g.skey, reinterpret_cast<int *>(g.stats_d + 4));
+               refine ? nullptr : g.sq, g.skey, (unsigned long long *)(g.stats_d + 4));
     launch_pdl(k_bucket_colscan, (K + 31) / 32, 32 * kColWarps, 0, stream, K, ctas, g.hist, g.base);
     launch_pdl(k_bucket_base, 1, 1024, 0, stream, bp, g.base);
     // windows of ~equal expected slot counts (refine: equal-size buckets; coarse: cost-weighted

@@ -191,6 +191,9 @@ struct SortedView {
     const uint32_t *__restrict__ slot;   // lookup offset (i - first) of sorted slot j
     const uint32_t *__restrict__ mb_dev; // device copy of matbase (fused path)
     int *work;                           // fused path: work-chunk counter (zeroed per chunk)
+    unsigned int *done;                  // S, last chunk: CTAs finished (zeroed with work)
+    unsigned long long *pub;             // S, last chunk: host-mapped {hash, pairs} written by
+                                         // the last CTA (no device-to-host copy), else null
     uint32_t matbase[kMaterials + 1];    // split path: first slot of each material; [12] = count
 };
 
