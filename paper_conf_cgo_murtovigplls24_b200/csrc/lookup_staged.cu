@@ -1,9 +1,10 @@
 // lookup_staged.cu -- XS_SEARCH_S: the sorted lookup kernel with staged warp windows
-// (DESIGN.md §6.5c).  Same work queue as k_lookup (lookup_fused.cu): each warp pulls chunks
-// of 4 x 32 consecutive sorted slots.  Per iteration a warp takes 32 lookups; for each
-// material among them (in sorted order almost always one) the lanes of that material form
-// the window [q_lo, q_hi] and every nuclide of the material is resolved through a window
-// of interval records staged in shared memory.
+// (DESIGN.md §6.5c).  A persistent grid (2 CTAs of 256 threads per SM); each warp pulls work
+// chunks of kStChunk = 256 consecutive sorted slots from an atomic counter and takes
+// 32 x kLpl = 128 of them (4 per lane) per iteration; for each material among them (in
+// sorted order almost always one) the lanes of that material form the window [q_lo, q_hi]
+// and every nuclide of the material is resolved through a window of interval records staged
+// in shared memory.
 #include <algorithm>
 
 #include "lookup_common.cuh"
