@@ -159,7 +159,13 @@ def cpu_baseline(w, lookups_cap: int, seconds: float):
     t0 = time.perf_counter()
     r = P.run_range(LOOKUP_SEED, 0, n, macro=False)
     dt = time.perf_counter() - t0
+    # plus one single-thread run (a ~1/threads-sized sample, same rate basis)
+    n1 = max(1000, n // max(threads, 1))
+    t0 = time.perf_counter()
+    P.run_range(LOOKUP_SEED, 0, n1, macro=False, threads=1)
+    dt1 = time.perf_counter() - t0
     return {"value": n / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "single_thread": {"value": n1 / dt1, "unit": UNIT, "sample": f"lookups [0, {n1})"},
             "sample": f"lookups [0, {n}) of {w.name} ({w.n_nuclides}x{w.n_gridpoints} "
                       f"{GRID_NAMES[w.grid_type]}), OpenMP static over lookups, {dt:.1f} s wall "
                       f"(grid build {setup_s:.1f} s untimed)",
