@@ -156,6 +156,22 @@ __device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, do
         return search<SEARCH>(Ei, 0, gv.n - 1, q);
     } else if constexpr (GRID == XS_UNIONIZED) {
         return __ldg(gv.IDX + (size_t)e_union * (uint32_t)gv.n_nuc + nuc);
+    } else if constexpr (kHashFast && (SEARCH == XS_SEARCH_H || SEARCH == XS_SEARCH_S)) {
+        // R7's window by a shorter dependent chain (H and S only; the paper's variants keep
+        // R7 as written).  Any bin b in range gives L(q) exactly: Listing 1 on [lo, hi] returns
+        // L(q) whenever E[lo] <= q < E[hi] (or hi = n-1), and the guards send every other q to
+        // the full search -- so b comes from a multiply instead of the IEEE division (they
+        // differ only where RN(q bins) and RN(q / du) straddle an integer), and the two guard
+        // energies are loaded alongside the window search instead of before it.
+        int64_t b = (int64_t)__dmul_rn(q, (double)gv.bins);
+        b = b < 0 ? 0 : (b > gv.bins - 1 ? gv.bins - 1 : b);
+        const int lo = __ldg(gv.H + b * gv.n_nuc + nuc);
+        const int hi = (b == gv.bins - 1) ? gv.n - 1 : __ldg(gv.H + (b + 1) * gv.n_nuc + nuc) + 1;
+        const double e_lo = __ldg(Ei + lo), e_hi = __ldg(Ei + hi);
+        int L = search<SEARCH>(Ei, lo, hi, q);
+        if (q < e_lo || (hi < gv.n - 1 && q >= e_hi))
+            L = search<SEARCH>(Ei, 0, gv.n - 1, q);
+        return L;
     } else { // hash window with guards (R7)
         int64_t b = (int64_t)__ddiv_rn(q, gv.du);
         b = b < 0 ? 0 : (b > gv.bins - 1 ? gv.bins - 1 : b);

@@ -38,6 +38,12 @@ constexpr int kMaxEnergyBins = 4096;
 #endif
 // XS_IV: lookups interpolate from per-interval records (iv) instead of point pairs (pts)
 constexpr bool kIv = XS_IV;
+#ifndef XS_HASH_FAST
+#define XS_HASH_FAST 1
+#endif
+// XS_HASH_FAST: H and S find the hash-grid window with a multiply and overlapped guard loads
+// (lookup_common.cuh lower_index; 0 = R7 as written, for the A/B)
+constexpr bool kHashFast = XS_HASH_FAST;
 constexpr int kTreeFan = 16;     // separator keys per node: one 128 B line
 constexpr int kTreeMaxLevels = 6; // n < 17^6 * 16 for every n_gridpoints < 2^31
 
