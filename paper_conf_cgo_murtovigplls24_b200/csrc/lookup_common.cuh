@@ -168,7 +168,7 @@ __device__ __forceinline__ int lower_index(const GridView &gv, const Row &rw, do
         const int lo = __ldg(gv.H + b * gv.n_nuc + nuc);
         const int hi = (b == gv.bins - 1) ? gv.n - 1 : __ldg(gv.H + (b + 1) * gv.n_nuc + nuc) + 1;
         const double e_lo = __ldg(Ei + lo), e_hi = __ldg(Ei + hi);
-        int L = search<SEARCH>(Ei, lo, hi, q);
+        int L = kHashK4 ? search_K4(Ei, lo, hi, q) : search<SEARCH>(Ei, lo, hi, q);
         if (q < e_lo || (hi < gv.n - 1 && q >= e_hi))
             L = search<SEARCH>(Ei, 0, gv.n - 1, q);
         return L;

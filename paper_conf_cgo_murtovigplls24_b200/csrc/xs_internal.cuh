@@ -44,6 +44,11 @@ constexpr bool kIv = XS_IV;
 // XS_HASH_FAST: H and S find the hash-grid window with a multiply and overlapped guard loads
 // (lookup_common.cuh lower_index; 0 = R7 as written, for the A/B)
 constexpr bool kHashFast = XS_HASH_FAST;
+#ifndef XS_HASH_K4
+#define XS_HASH_K4 1
+#endif
+// XS_HASH_K4: that window searched 4-ary (search.cuh search_K4); 0 = Listing 1 (M)
+constexpr bool kHashK4 = XS_HASH_K4;
 constexpr int kTreeFan = 16;     // separator keys per node: one 128 B line
 constexpr int kTreeMaxLevels = 6; // n < 17^6 * 16 for every n_gridpoints < 2^31
 
