@@ -110,7 +110,7 @@ __device__ __forceinline__ int bin_lower(const double *__restrict__ A, const Bin
 {
     if (bn.cnt <= 1)
         return bn.lo + ((bn.cnt == 1 && bn.e_next <= q) ? 1 : 0);
-    return search<XS_SEARCH_U2>(A, bn.lo, bn.lo + bn.cnt + 1, q);
+    return kBinK4 ? search_K4(A, bn.lo, bn.lo + bn.cnt + 1, q) : search<XS_SEARCH_U2>(A, bn.lo, bn.lo + bn.cnt + 1, q);
 }
 
 // 48 B NucRef as three 16 B broadcast loads (fields a kernel does not use are dead code)

@@ -49,6 +49,11 @@ constexpr bool kHashFast = XS_HASH_FAST;
 #endif
 // XS_HASH_K4: that window searched 4-ary (search.cuh search_K4); 0 = Listing 1 (M)
 constexpr bool kHashK4 = XS_HASH_K4;
+#ifndef XS_BIN_K4
+#define XS_BIN_K4 1
+#endif
+// XS_BIN_K4: the bin windows of H and S (nuclide and unionized grids) searched 4-ary too; 0 = U2
+constexpr bool kBinK4 = XS_BIN_K4;
 constexpr int kTreeFan = 16;     // separator keys per node: one 128 B line
 constexpr int kTreeMaxLevels = 6; // n < 17^6 * 16 for every n_gridpoints < 2^31
 
