@@ -26,6 +26,9 @@
 namespace xs {
 
 constexpr int kSortTpb = 1024;
+#ifndef XS_SCATTER_VEC
+#define XS_SCATTER_VEC 1
+#endif
 constexpr int64_t kScatterWindow = int64_t(48) << 20; // max bytes of slots one scatter launch writes
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
@@ -215,6 +218,37 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int
     // 4 keys in flight per thread, then their shared-memory atomics and 4 B stores
     // (recording each lookup's rank in the count pass to drop the atomics was measured
     // slower)
+#if XS_SCATTER_VEC
+    // 8 keys per 16 B load (per_cta is a multiple of 8, so the chunk is 16 B aligned), two
+    // loads in flight per thread; a thread's 8 lookups are consecutive offsets (any order
+    // inside a bucket is valid)
+    const int nvec = max(0, end - beg) >> 3;
+    const uint4 *kv = reinterpret_cast<const uint4 *>(key_of + beg);
+    auto put = [&](uint32_t w, int j0) {
+        const uint32_t k0 = w & 0xffffu, k1 = w >> 16;
+        if (k0 - (uint32_t)klo < span)
+            slot_of[atomicAdd(&sh[k0], 1u)] = (uint32_t)j0;
+        if (k1 - (uint32_t)klo < span)
+            slot_of[atomicAdd(&sh[k1], 1u)] = (uint32_t)(j0 + 1);
+    };
+    int v = threadIdx.x;
+    for (; v + kSortTpb < nvec; v += 2 * kSortTpb) {
+        const uint4 a = __ldg(kv + v), b = __ldg(kv + v + kSortTpb);
+        const int ja = beg + 8 * v, jb = ja + 8 * kSortTpb;
+        put(a.x, ja); put(a.y, ja + 2); put(a.z, ja + 4); put(a.w, ja + 6);
+        put(b.x, jb); put(b.y, jb + 2); put(b.z, jb + 4); put(b.w, jb + 6);
+    }
+    for (; v < nvec; v += kSortTpb) {
+        const uint4 a = __ldg(kv + v);
+        const int ja = beg + 8 * v;
+        put(a.x, ja); put(a.y, ja + 2); put(a.z, ja + 4); put(a.w, ja + 6);
+    }
+    for (int j = beg + 8 * nvec + threadIdx.x; j < end; j += kSortTpb) {
+        const uint32_t k = key_of[j];
+        if (k - (uint32_t)klo < span)
+            slot_of[atomicAdd(&sh[k], 1u)] = (uint32_t)j;
+    }
+#else
     int j = beg + threadIdx.x;
     for (; j + 3 * kSortTpb < end; j += 4 * kSortTpb) {
         uint32_t kk[4];
@@ -231,6 +265,7 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int
         if (k - (uint32_t)klo < span)
             slot_of[atomicAdd(&sh[k], 1u)] = (uint32_t)j;
     }
+#endif
 }
 
 __global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of, const double *__restrict__ q_of,
@@ -523,7 +558,7 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     *K_out = K;
     const int sms = sm_count_dev();
     const int ctas = (int)std::max<int64_t>(1, std::min<int64_t>(sms, (cn + kSortTpb - 1) / kSortTpb));
-    const int per_cta = (int)((cn + ctas - 1) / ctas);
+    const int per_cta = (int)(((cn + ctas - 1) / ctas + 7) / 8 * 8); // 16 B aligned key chunks
     ensure_sort_space(g, cn, ctas, K);
     const Affine J = lcg_jump(2 * (uint64_t)kSortTpb);
     const size_t smem = (size_t)K * 4;
