@@ -29,7 +29,7 @@ constexpr int kSortTpb = 1024;
 #ifndef XS_SCATTER_VEC
 #define XS_SCATTER_VEC 1
 #endif
-constexpr int64_t kScatterWindow = int64_t(48) << 20; // max bytes of slots one scatter launch writes
+constexpr int64_t kScatterWindow = int64_t(64) << 20; // max bytes of slots one scatter launch writes
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
                                                             uint32_t *__restrict__ hist, double *__restrict__ q_of,
@@ -569,10 +569,10 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     launch_pdl(k_bucket_base, 1, 1024, 0, stream, bp, g.base);
     // windows of ~equal expected slot counts (refine: equal-size buckets; coarse: cost-weighted
     // buckets, so the windows are only approximately equal)
-    // window: 1/8 of the slot array, within [16, 48] MB -- more windows keep each one's
+    // window: 1/6 of the slot array, within [16, 64] MB -- more windows keep each one's
     // random writes more L2-local, but every window re-reads all 2 B keys (measured: 17M
-    // lookups best at 16 MB, 100M-125M at 48 MB)
-    int64_t win_bytes = std::min<int64_t>(kScatterWindow, std::max<int64_t>(int64_t(16) << 20, cn * 4 / 8));
+    // lookups best at 16 MB, 100M-125M at 48 MB; with the 16 B key loads at 64 MB, r01be)
+    int64_t win_bytes = std::min<int64_t>(kScatterWindow, std::max<int64_t>(int64_t(16) << 20, cn * 4 / 6));
     if (const char *env = std::getenv("XS_SCATTER_WINDOW_MB"))
         win_bytes = std::max(1ll, std::atoll(env)) << 20;
     int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, (cn * 4 + win_bytes - 1) / win_bytes));
