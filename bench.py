@@ -1,28 +1,40 @@
 #!/usr/bin/env python
-"""bench.py -- lookups/s of the XSBench-style macroscopic XS lookup on B200.
+"""bench.py -- lookups/s of the XSBench-style macroscopic XS lookup on 1..8 B200.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--workload small] [--search U4] [--sort material_energy]
+                    [--workload large-U] [--scaling strong|weak] [--search S]
+                    [--workloads small,large,XL]
 
 One step = one pass of the whole hot path (sampling,
-(material, energy) ordering, search, interpolation, accumulation, verification) over
-one batch of lookups on every rank, inputs (the grid) resident in HBM.  Weak scaling:
-rank r owns lookups [r*L, (r+1)*L) of each batch (L = the workload's per-GPU count).
-Rank 0 prints ONE JSON line.  Timing: W untimed warm-up steps, then K steps, each
-bracketed by CUDA events on the launching stream with the 126 MB L2 flushed (a
-256 MiB write) before it, outside the events; barrier + synchronize on both sides;
-the max over ranks of the summed step times.  Grid creation is untimed (XSBench's
-grid_init_do_not_profile [XSB]).
+(material, energy) ordering, search, interpolation, accumulation, verification) over one
+batch of lookups on every rank, the grid resident in HBM.  With --gpus N > 1 and no
+torchrun environment, bench.py re-launches itself under torch.distributed.run with one
+process per GPU; XS_DIST_BACKEND=gloo runs the ranks over gloo instead of
+NCCL (ranks share the visible GPUs round-robin, so a 1-GPU box can run 2 ranks).
 
---impl reference times the CPU oracle (oracle/, plain C + OpenMP) on the box's host
-cores on a bounded sample of the same workload (rank 0 only).
+Scaling: strong (the default except XL) splits the workload's fixed total
+into rank ranges [floor(rT/N), floor((r+1)T/N)); weak gives every rank its own block of
+the workload's per-rank count (XL: 125M per rank, so N = 8 is exactly the 1B-lookup
+configuration of BASELINE.json configs[4]).  Counter-based sampling makes the results
+independent of the split; every rank's hash is checked against the CPU oracle's golden
+hashes (tests/golden/hashes.json, written by tools/oracle_golden.py from oracle/ only).
+
+Timing: W untimed warm-up steps, then K steps, each bracketed by CUDA events on the
+launching stream with the L2 flushed (a 256 MiB write) before it, outside the events;
+barrier + synchronize on both sides; value = lookups of all ranks / the max over ranks of
+the summed step times.  Grid creation is untimed (XSBench's grid_init_do_not_profile).
+
+--impl reference times the CPU oracle (oracle/, plain C + OpenMP) on the box's host cores
+on a bounded sample of the same workload (rank 0 only).
 """
 from __future__ import annotations
 
 import argparse
+import hashlib
 import json
 import math
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -36,17 +48,28 @@ from xs_workloads import GRID_SEED, LOOKUP_SEED, MEAN_NUCS, WORKLOADS, GRID_NAME
 METRIC = "lookups/sec (device-timed, max over ranks)"
 UNIT = "lookups/s"
 L2_FLUSH_BYTES = 256 << 20
-BYTES_PER_PAIR = 96  # two 48 B point records per (lookup, nuclide)
+BYTES_PER_PAIR = 96      # two 48 B point records per (lookup, nuclide)
+POINT_RECORD_BYTES = 48  # {E, 5 channels} fp64 per grid point
+STREAM_BYTES = 12        # sorted slot (u32) + energy (f64) per lookup, read by the lookup kernel
+# FP64 flops per (lookup, nuclide) pair that any bit-exact evaluation of reading R8 must
+# execute, with d = E_hi - E_lo, y = RN(1/d) and dX_c precomputed:
+# a = E_hi - q (1), Markstein's quotient q0 = a y, r = fma(-d, q0, a), f = fma(r, y, q0)
+# (1 + 2 + 2), micro_c = fma(-f, dX_c, X_c) (5 x 2), acc_c = fma(micro_c, conc, acc_c) (5 x 2)
+FLOPS_PER_PAIR = 26
+FP64_LANES_PER_SM = 64   # B200: 64 FP64 FMA lanes per SM per clock
+GOLDEN = os.path.join(ROOT, "tests", "golden", "hashes.json")
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--workload", default="small", choices=sorted(WORKLOADS))
-    p.add_argument("--lookups", type=int, default=0, help="override lookups per GPU")
+    p.add_argument("--workload", default="large-U", choices=sorted(WORKLOADS))
+    p.add_argument("--scaling", default="", choices=["", "strong", "weak"],
+                   help="default: the workload's (XL weak at 125M per rank, the rest strong)")
+    p.add_argument("--lookups", type=int, default=0, help="override: job total (strong) or per rank (weak)")
     p.add_argument("--search", default="S")
     p.add_argument("--sort", default="material_energy")
     p.add_argument("--energy-bins", type=int, default=0)
@@ -55,14 +78,33 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--ab", default="M,U1,U2,U4,U8,B,W,H,S", help="search variants for the A/B sub-object ('' = off)")
     p.add_argument("--ab-steps", type=int, default=5)
+    p.add_argument("--workloads", default="small,large,XL",
+                   help="other configurations measured into the `workloads` sub-object ('' = off)")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="target wall time of the CPU sample")
-    return p.parse_args()
+    return p.parse_args(argv)
+
+
+# ------------------------------------------------------------------ sizes and rooflines
+def scaling_of(a, w) -> str:
+    return a.scaling or w.scaling
+
+
+def rank_range(w, scaling: str, total_override: int, rank: int, world: int):
+    """(first, count) of this rank."""
+    from paper_conf_cgo_murtovigplls24_b200 import driver
+    n = total_override or w.lookups
+    return driver.shard(n, rank, world) if scaling == "strong" else driver.weak_range(n, rank)
+
+
+def job_lookups(w, scaling: str, total_override: int, world: int) -> int:
+    n = total_override or w.lookups
+    return n if scaling == "strong" else n * world
 
 
 def algorithmic_bytes_per_lookup(w) -> float:
-    """the useful bytes of a random gather -- E[n_nuc] x 96 B (nuclide),
+    """the useful bytes of a RANDOM gather -- E[n_nuc] x 96 B (nuclide),
     + 4 B of IDX per pair (unionized), + 8*ceil(log2(W+1)) B of window probes (hash).
-    Probes into L2-resident search arrays are excluded."""
+    Valid for XSBench's unsorted order only."""
     m = MEAN_NUCS[68 if w.n_nuclides == 68 else 355]
     if w.grid_type == 1:
         per_pair = BYTES_PER_PAIR
@@ -74,7 +116,16 @@ def algorithmic_bytes_per_lookup(w) -> float:
     return m * per_pair
 
 
-def measured_peaks():
+def hbm_min_bytes(w, lookups: int) -> float:
+    """A lower bound on the DRAM bytes one lookup-kernel launch over `lookups` sorted lookups
+    must move: every point record once (at these sizes every interval of
+    every nuclide is visited: >= 2.4M lookups per fuel nuclide per launch) plus the sorted
+    (slot, energy) stream.  Search structures (E, bins, U, IDX, H) are left out, so the
+    fraction is an underestimate."""
+    return w.n_points * POINT_RECORD_BYTES + STREAM_BYTES * lookups
+
+
+def measured_hbm_peak():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             d = json.load(f)
@@ -83,17 +134,111 @@ def measured_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def fp64_peak_tflops(sms: int):
+    """FP64 peak: the guide's unit count (64 FMA lanes/SM/clk) x 2 flops x SMs x max SM clock;
+    profiles/fp64_peak.json (tools/fp64_peak.cu, a DFMA microbenchmark on this pool's B200)
+    when present."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "fp64_peak.json")) as f:
+            d = json.load(f)
+        return float(d["tflops"]), "measured (profiles/fp64_peak.json: DFMA microbenchmark)"
+    except Exception:
+        mhz = 1965.0
+        try:
+            with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+                mhz = float(json.load(f).get("sm_max_mhz", mhz))
+        except Exception:
+            pass
+        return sms * FP64_LANES_PER_SM * 2 * mhz * 1e6 / 1e12, \
+            f"derived: {sms} SMs x {FP64_LANES_PER_SM} FP64 lanes x 2 flops x {mhz:.0f} MHz"
+
+
+def libxs_sha() -> str:
+    try:
+        from paper_conf_cgo_murtovigplls24_b200 import _xs
+        with open(_xs.LIB_PATH, "rb") as f:
+            return hashlib.sha256(f.read()).hexdigest()[:16]
+    except Exception:
+        return ""
+
+
 def ncu_record(workload: str, search: str, sort: str):
-    """The committed ncu --set full capture of k_lookup for this configuration
-    (profiles/ncu_traffic.json: DRAM bytes and warp instructions per launch)."""
+    """The committed ncu --set full capture of this configuration's lookup kernel
+    (profiles/ncu_traffic.json), used only if it was taken on THIS libxs.so build."""
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
             d = json.load(f)
-        return d.get(f"{workload}/{search}/{sort}")
+        rec = d.get(f"{workload}/{search}/{sort}")
+        if rec and rec.get("libxs_sha") == libxs_sha():
+            return rec
+    except Exception:
+        pass
+    return None
+
+
+def roofline(w, search, sort, lookups, pairs, kernel_ms, sms, clocks=None, with_ncu=True):
+    """The lookup kernel against what the work needs: FP64 flops (alu) and
+    the HBM minimum; `bound` is whichever fraction is higher.  SURVEY.md §8d's random-gather
+    bytes are kept as `random_gather_equiv` (valid as a roofline for unsorted order only)."""
+    sec = kernel_ms / 1e3
+    hbm_peak, hbm_src = measured_hbm_peak()
+    fp_peak, fp_src = fp64_peak_tflops(sms)
+    flops = FLOPS_PER_PAIR * pairs
+    alu = {"achieved": flops / sec / 1e12, "peak": fp_peak, "unit": "TFLOP/s",
+           "frac": flops / sec / 1e12 / fp_peak, "flops_per_pair": FLOPS_PER_PAIR, "pairs": pairs,
+           "peak_source": fp_src}
+    hb = hbm_min_bytes(w, lookups)
+    hbm = {"achieved": hb / sec / 1e9, "peak": hbm_peak, "unit": "GB/s", "frac": hb / sec / 1e9 / hbm_peak,
+           "bytes_per_launch": hb, "peak_source": hbm_src}
+    rg_b = algorithmic_bytes_per_lookup(w) * lookups
+    rg = {"achieved": rg_b / sec / 1e9, "unit": "GB/s", "bytes_per_lookup": algorithmic_bytes_per_lookup(w),
+          "frac_of_hbm": rg_b / sec / 1e9 / hbm_peak}
+    try:
+        with open(os.path.join(ROOT, "profiles", "l2_gather.json")) as f:
+            lg = json.load(f)
+        key = {"small": "small_points_37MB", "large": "large_points_193MB", "large-U": "large_points_193MB",
+               "XL": "xl_points_4.07GB"}.get(w.name)
+        if key and lg["gathers"].get(key):
+            gp = lg["gathers"][key]["GBps_useful"]
+            rg.update(measured_gather_peak=gp, frac_of_measured_gather=rg_b / sec / 1e9 / gp, buffer=key)
+    except Exception:
+        pass
+    rg["note"] = ("SURVEY.md §8d random-gather bytes; in (material, energy) order warps share their grid "
+                  "points, so this exceeds any bandwidth and is not a roofline there")
+    kernel = "k_lookup_staged" if search == "S" and sort in ("material_energy", "material") else "k_lookup"
+    top = alu if alu["frac"] >= hbm["frac"] else hbm
+    line = {"bound": "alu" if top is alu else "hbm", "kernel": kernel, "achieved": top["achieved"],
+            "peak": top["peak"], "unit": top["unit"], "frac": top["frac"], "traffic": None,
+            "alu_fp64": alu, "hbm_min": hbm, "random_gather_equiv": rg}
+    rec = ncu_record(w.name, search, sort) if with_ncu else None
+    if rec:
+        line["traffic"] = rec["dram_bytes_per_launch"] * lookups / rec.get("lookups", lookups)
+        line["ncu"] = {k: rec.get(k) for k in ("libxs_sha", "report", "round", "dram_bytes_per_launch",
+                                               "l2_hit_pct", "l1_hit_pct", "sectors_per_request",
+                                               "lsu_wavefronts_pct_of_peak", "fp64_pipe_pct", "issue_active_pct",
+                                               "branch_uniform_pct")}
+        line["hbm_min"]["refetch"] = rec["dram_bytes_per_launch"] / hb
+    else:
+        line["ncu"] = {"note": "no ncu capture of this libxs.so build for this configuration"}
+    return line
+
+
+def golden_expect(name: str, first: int, count: int):
+    """The oracle's hash / pairs over [first, first + count) when the range is a union of the
+    golden eighths (tests/golden/hashes.json), else None."""
+    try:
+        with open(GOLDEN) as f:
+            g = json.load(f)[name]
     except Exception:
         return None
+    b = g["bounds"]
+    if first not in b or (first + count) not in b:
+        return None
+    i, j = b.index(first), b.index(first + count)
+    return sum(g["hash"][i:j]), sum(g["pairs"][i:j])
 
 
+# ------------------------------------------------------------------ clocks
 class Clocks:
     """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
@@ -144,6 +289,15 @@ class Clocks:
                 "samples": len(rows)}
 
 
+# ------------------------------------------------------------------ the reference arm
+def config_of(a, w, world: int) -> dict:
+    """The workload `config` both arms print (identical, so the driver can pair them)."""
+    sc = scaling_of(a, w)
+    return {"workload": w.name, "n_nuclides": w.n_nuclides, "n_gridpoints": w.n_gridpoints,
+            "grid": GRID_NAMES[w.grid_type], "lookups_total": job_lookups(w, sc, a.lookups, world),
+            "scaling": sc, "l2_flush": not a.no_flush, "parallelism": f"dp{world} (lookup index ranges)"}
+
+
 def cpu_baseline(w, lookups_cap: int, seconds: float):
     """The oracle as it stands on this host's cores: a bounded sample of the workload."""
     import oracle
@@ -173,11 +327,11 @@ def cpu_baseline(w, lookups_cap: int, seconds: float):
 
 
 def run_reference(a, w):
-    """--impl reference: the oracle as the reference arm (rank 0 only)."""
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
+    """--impl reference: the oracle as the reference arm (rank 0 only; other ranks exit 0)."""
+    if int(os.environ.get("RANK", "0")) != 0:
         return
     import oracle
+    world = int(os.environ.get("WORLD_SIZE", str(a.gpus)))
     P = oracle.Problem(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED, build_idx=False)
     threads = oracle.max_threads()
     n = 20_000
@@ -185,214 +339,244 @@ def run_reference(a, w):
     P.run_range(LOOKUP_SEED, 0, n, macro=False)
     rate = n / max(time.perf_counter() - t0, 1e-6)
     budget = 150.0 / max(a.steps + a.warmup, 1)  # whole run within a few minutes
-    n = int(max(10_000, min(w.lookups, rate * budget)))
+    total = job_lookups(w, scaling_of(a, w), a.lookups, world)
+    n = int(max(10_000, min(total, rate * budget)))
     times = []
     for k in range(a.warmup + a.steps):
         t0 = time.perf_counter()
         P.run_range(LOOKUP_SEED, 0, n, macro=False)
         if k >= a.warmup:
             times.append(time.perf_counter() - t0)
-    total = sum(times)
-    value = n * len(times) / total
+    tsum = sum(times)
+    value = n * len(times) / tsum
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": a.gpus,
-        "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * total / len(times),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * tsum / len(times),
+        "higher_is_better": True, "scaling": scaling_of(a, w), "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (XSBench LCG grid + lookups, seeds 42/1070)",
-        "config": {"workload": w.name, "n_nuclides": w.n_nuclides, "n_gridpoints": w.n_gridpoints,
-                   "grid": GRID_NAMES[w.grid_type], "lookups_per_step": n},
+        "config": config_of(a, w, world),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
-                         "sample": f"lookups [0, {n}) of {w.name} per step"},
+                         "sample": f"lookups [0, {n}) of {w.name} per step (the job's {total} lookups "
+                                   f"bounded to ~{budget:.0f} s of CPU work per step), host cores only"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
-def run_ours(a, w):
-    import torch
-    import paper_conf_cgo_murtovigplls24_b200 as xs
-    from paper_conf_cgo_murtovigplls24_b200 import driver
+# ------------------------------------------------------------------ our arm
+class Runner:
+    """One grid on this rank's GPU and the timed-step protocol."""
 
-    R = driver.init()
-    dev = torch.device("cuda", torch.cuda.current_device())
-    L = a.lookups or w.lookups
-    first, count = driver.weak_range(L, R.rank)
-    g = xs.Grid(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED)
-    assert driver.replicas_identical(g.checksum()), "grid replicas differ across ranks"
-    stream = torch.cuda.current_stream()
-    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
-    opts = dict(search=a.search, sort=a.sort, energy_bins=a.energy_bins, timing=True)
+    def __init__(self, a, w, R, scaling):
+        import torch
+        import paper_conf_cgo_murtovigplls24_b200 as xs
+        from paper_conf_cgo_murtovigplls24_b200 import driver
+        self.torch, self.xs, self.driver, self.a, self.w, self.R = torch, xs, driver, a, w, R
+        self.scaling = scaling
+        self.first, self.count = rank_range(w, scaling, a.lookups, R.rank, R.world)
+        self.total = int(driver.sum_over_ranks(self.count))
+        self.g = xs.Grid(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED)
+        assert driver.replicas_identical(self.g.checksum()), "grid replicas differ across ranks"
+        self.stream = torch.cuda.current_stream()
+        self.flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=self.g.device)
+        self.opts = dict(search=a.search, sort=a.sort, energy_bins=a.energy_bins, timing=True)
 
-    def step(**o):
-        return g.lookup_range(first, count, LOOKUP_SEED, None, **{**opts, **o})
+    def step(self, **o):
+        return self.g.lookup_range(self.first, self.count, LOOKUP_SEED, None, **{**self.opts, **o})
 
-    def timed_steps(k_steps, **o):
+    def timed(self, k_steps, warm, **o):
+        torch = self.torch
+        for _ in range(warm):
+            self.step(**o)
+        self.driver.barrier()
+        torch.cuda.synchronize()
         evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(k_steps)]
         out = []
         for k in range(k_steps):
-            if not a.no_flush:
-                flush.fill_(k)
-            evs[k][0].record(stream)
-            out.append(step(**o))
-            evs[k][1].record(stream)
+            if not self.a.no_flush:
+                self.flush.fill_(k)
+            evs[k][0].record(self.stream)
+            out.append(self.step(**o))
+            evs[k][1].record(self.stream)
         torch.cuda.synchronize()
-        return [s_.elapsed_time(e_) for s_, e_ in evs], out
+        self.driver.barrier()
+        ms = [s_.elapsed_time(e_) for s_, e_ in evs]
+        return ms, out, self.driver.max_over_ranks(sum(ms))
 
-    ref_stats = None
-    for _ in range(a.warmup):
-        ref_stats = step()
-    driver.barrier()
-    torch.cuda.synchronize()
+    def golden(self, stats):
+        """Every rank's hash and pairs against the oracle's golden eighths; True/False/None
+        (None: the split does not fall on the golden boundaries)."""
+        exp = golden_expect(self.w.name, self.first, self.count)
+        ok = -1 if exp is None else int(stats.hash == exp[0] and stats.pairs == exp[1])
+        lo = self.driver.min_over_ranks(ok)
+        return None if lo < 0 else bool(lo)
+
+    def close(self):
+        self.g.close()
+
+
+def summarize(run: Runner, ms_max, stats, steps, sms, clocks=None, **o):
+    s0 = stats[0]
+    h, nl, npairs, _ = run.driver.reduce_stats(s0.hash, s0.lookups, s0.pairs, 0.0)
+    lookup_ms = statistics.mean(x.lookup_ms for x in stats)
+    search = o.get("search", run.a.search)
+    sort = o.get("sort", run.a.sort)
+    return {"value": run.total * steps / (ms_max / 1e3), "ms_per_step": ms_max / steps,
+            "lookups_per_gpu": run.count, "sort_ms": statistics.mean(x.sample_ms for x in stats),
+            "lookup_ms": lookup_ms, "hash": h, "pairs": npairs, "lookups": nl,
+            "hash_consistent": all(x.hash == s0.hash for x in stats),
+            "golden_match": run.golden(s0),
+            "roofline": roofline(run.w, search, sort, run.count, s0.pairs, lookup_ms, sms, clocks)}
+
+
+def run_ours(a, w):
+    import torch
+    from paper_conf_cgo_murtovigplls24_b200 import driver
+
+    R = driver.init(backend=os.environ.get("XS_DIST_BACKEND") or None)
+    if R.world != a.gpus:
+        raise SystemExit(f"bench.py: --gpus {a.gpus} but WORLD_SIZE={R.world}")
+    dev = torch.device("cuda", torch.cuda.current_device())
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    scaling = scaling_of(a, w)
+    run = Runner(a, w, R, scaling)
+
     with Clocks(torch.cuda.current_device()) as clk:
-        step_ms, stats = timed_steps(a.steps)
-    driver.barrier()
-    total_ms = driver.max_over_ranks(sum(step_ms))
-    lookup_ms = [s.lookup_ms for s in stats]
-    hashes = {s.hash for s in stats}
-    assert len(hashes) == 1 and (ref_stats is None or ref_stats.hash in hashes), "non-deterministic hash"
-    h, nl, npairs, _ = driver.reduce_stats(stats[0].hash, stats[0].lookups, stats[0].pairs, 0.0)
+        step_ms, stats, total_ms = run.timed(a.steps, a.warmup)
+    clocks = clk.summary()
+    assert len({s.hash for s in stats}) == 1, "non-deterministic hash"
+    main = summarize(run, total_ms, stats, a.steps, sms)
+
+    # ---- the north-star quantity: the unmerged (u&u, u=2) Listing-1 search, same config and N
+    north = {}
+    for label, o in (("U2 (material, energy) order", dict(search="U2")),
+                     ("U2 XSBench order (unsorted)", dict(search="U2", sort="none"))):
+        ms, sts, mx = run.timed(a.ab_steps, 2, **o)
+        north[label] = summarize(run, mx, sts, a.ab_steps, sms, **o)
+        north[label]["hash_ok"] = all(x.hash == stats[0].hash for x in sts)
 
     # ---- the paper's A/B on this workload: every search variant, same protocol, fewer steps
     ab = {}
-    for v in [x for x in a.ab.split(",") if x]:
-        for _ in range(2):
-            step(search=v)
-        ms, sts = timed_steps(a.ab_steps, search=v)
-        ms_max = driver.max_over_ranks(sum(ms))
-        ab[v] = {"value": R.world * count * a.ab_steps / (ms_max / 1e3),
-                 "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
-    if a.ab:
-        for _ in range(2):
-            step(search="H", sort="history")
-        ms, sts = timed_steps(a.ab_steps, search="H", sort="history")
-        ms_max = driver.max_over_ranks(sum(ms))
-        ab["H/history (XSBench history order, 34 lookups/particle)"] = {
-            "value": R.world * count * a.ab_steps / (ms_max / 1e3),
-            "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
-        for _ in range(2):
-            step(coarse=True)
-        ms, sts = timed_steps(a.ab_steps, coarse=True)
-        ms_max = driver.max_over_ranks(sum(ms))
-        ab[f"{a.search}/coarse (bucket order without the k_bucket_refine pass)"] = {
-            "value": R.world * count * a.ab_steps / (ms_max / 1e3), "sort_ms": statistics.mean(x.sample_ms for x in sts),
-            "lookup_ms": statistics.mean(x.lookup_ms for x in sts), "hash_ok": all(x.hash == stats[0].hash for x in sts)}
-        for _ in range(2):
-            step(search="M", sort="none")
-        ms, sts = timed_steps(a.ab_steps, search="M", sort="none")
-        ms_max = driver.max_over_ranks(sum(ms))
-        ab["M/unsorted (XSBench order)"] = {"value": R.world * count * a.ab_steps / (ms_max / 1e3),
-                                            "lookup_ms": statistics.mean(x.lookup_ms for x in sts),
-                                            "hash_ok": all(x.hash == stats[0].hash for x in sts)}
+    variants = [x for x in a.ab.split(",") if x]
+    extra = [("H/history (XSBench history order, 34 lookups/particle)", dict(search="H", sort="history")),
+             (f"{a.search}/coarse (bucket order without the k_bucket_refine pass)", dict(coarse=True)),
+             ("M/unsorted (XSBench order)", dict(search="M", sort="none"))] if variants else []
+    for label, o in [(v, dict(search=v)) for v in variants] + extra:
+        ms, sts, mx = run.timed(a.ab_steps, 2, **o)
+        ab[label] = {"value": run.total * a.ab_steps / (mx / 1e3), "sort_ms": statistics.mean(x.sample_ms for x in sts),
+                     "lookup_ms": statistics.mean(x.lookup_ms for x in sts),
+                     "hash_ok": all(x.hash == stats[0].hash for x in sts)}
 
     # ---- e2e: the public API with HOST output buffers (D2H of every macro XS in the region)
     e2e = None
     if not a.no_e2e:
-        host = torch.empty((count, 5), dtype=torch.float64).pin_memory()
+        host = torch.empty((run.count, 5), dtype=torch.float64).pin_memory()
         for _ in range(2):
-            g.lookup_range(first, count, LOOKUP_SEED, host, search=a.search, sort=a.sort)
+            run.g.lookup_range(run.first, run.count, LOOKUP_SEED, host, search=a.search, sort=a.sort)
         driver.barrier()
         torch.cuda.synchronize()
         t = []
         for k in range(max(3, a.steps // 4)):
             if not a.no_flush:
-                flush.fill_(k)
+                run.flush.fill_(k)
             torch.cuda.synchronize()
             t0 = time.perf_counter()
-            g.lookup_range(first, count, LOOKUP_SEED, host, search=a.search, sort=a.sort)
+            run.g.lookup_range(run.first, run.count, LOOKUP_SEED, host, search=a.search, sort=a.sort)
             t.append(time.perf_counter() - t0)
         e2e_s = driver.max_over_ranks(sum(t))
-        # the hash-only public call (XSBench's own result: the verification hash)
         th = []
         for k in range(max(3, a.steps // 4)):
             if not a.no_flush:
-                flush.fill_(k)
+                run.flush.fill_(k)
             torch.cuda.synchronize()
             t0 = time.perf_counter()
-            hh = xs.xs_lookup_batch(g.handle, count, LOOKUP_SEED, None) if R.world == 1 else \
-                g.lookup_range(first, count, LOOKUP_SEED, None, search=a.search, sort=a.sort).hash
+            if R.world == 1:
+                run.xs.xs_lookup_batch(run.g.handle, run.count, LOOKUP_SEED, None)
+            else:
+                run.g.lookup_range(run.first, run.count, LOOKUP_SEED, None, search=a.search, sort=a.sort)
             th.append(time.perf_counter() - t0)
         e2e_h = driver.max_over_ranks(sum(th))
-        e2e = {"value": R.world * count * len(t) / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 0,
-               "d2h_bytes_per_step": count * 5 * 8 + 16,
+        e2e = {"value": run.total * len(t) / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 0,
+               "d2h_bytes_per_step": run.count * 5 * 8 + 16,
                "note": "xs_lookup_range writing every macroscopic XS into pinned HOST memory (D2H "
-                       "overlapped with compute in 4M-lookup chunks), host wall clock; inputs are the "
-                       "(seed, range) scalars -- lookups are drawn on device by the method's "
-                       "counter-based LCG (DESIGN.md §8)",
-               "hash_only": {"value": R.world * count * len(th) / e2e_h, "d2h_bytes_per_step": 16,
-                             "call": "xs_lookup_batch (default options), host wall clock"}}
+                       "overlapped with compute in 4M-lookup chunks), host wall clock, max over ranks; "
+                       "inputs are the (seed, range) scalars -- lookups are drawn on device by the "
+                       "method's counter-based LCG (DESIGN.md §8)",
+               "hash_only": {"value": run.total * len(th) / e2e_h, "d2h_bytes_per_step": 16,
+                             "call": "xs_lookup_batch (default options) / xs_lookup_range, host wall clock"}}
+        del host
+
+    cb = None
+    if not a.no_cpu_baseline and R.world == 1:
+        cb = cpu_baseline(w, run.count, a.cpu_seconds)
+        gs = run.g.lookup_range(0, cb["_n"], LOOKUP_SEED, None, search=a.search, sort=a.sort)
+        cb["_match"] = bool(gs.hash == cb["_hash"])
+    run.close()
+    del run
+
+    # ---- the other configurations (sub-object), same protocol and N
+    workloads = {}
+    for name in [x for x in a.workloads.split(",") if x and x != w.name]:
+        ww = WORKLOADS[name]
+        sa = argparse.Namespace(**{**vars(a), "lookups": 0, "scaling": ""})
+        r2 = Runner(sa, ww, R, scaling_of(sa, ww))
+        ms, sts, mx = r2.timed(a.steps, a.warmup)
+        workloads[name] = {"config": config_of(sa, ww, R.world), **summarize(r2, mx, sts, a.steps, sms)}
+        r2.close()
+        del r2
+        torch.cuda.empty_cache()
 
     if R.rank != 0:
         driver.finalize()
         return
-    value = R.world * count * a.steps / (total_ms / 1e3)
-    peak, peak_src = measured_peaks()
-    bpl = algorithmic_bytes_per_lookup(w)
-    mean_lookup_ms = statistics.mean(lookup_ms)
-    achieved = bpl * count / (mean_lookup_ms / 1e3) / 1e9
-    rec = ncu_record(w.name, a.search, a.sort)
-    traffic = rec["dram_bytes_per_launch"] if rec else None
     line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": R.world, "steps": a.steps,
-        "warmup": a.warmup, "ms_per_step": total_ms / a.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "metric": METRIC, "value": main["value"], "unit": UNIT, "n_gpus": R.world, "steps": a.steps,
+        "warmup": a.warmup, "ms_per_step": main["ms_per_step"], "higher_is_better": True,
+        "scaling": scaling, "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (XSBench LCG grid + lookups, seeds 42/1070)",
-        "config": {"workload": w.name, "n_nuclides": w.n_nuclides, "n_gridpoints": w.n_gridpoints,
-                   "grid": GRID_NAMES[w.grid_type], "lookups_per_gpu": count, "search": a.search,
-                   "sort": a.sort, "l2_flush": not a.no_flush, "parallelism": f"dp{R.world} (index ranges)"},
+        "config": config_of(a, w, R.world),
+        "path": {"search": a.search, "sort": a.sort, "backend": driver.backend_name(),
+                 "lookups_per_gpu": main["lookups_per_gpu"]},
         "step_ms": {"median": statistics.median(step_ms), "rsd_pct": 100 * statistics.pstdev(step_ms) /
                     statistics.mean(step_ms), "min": min(step_ms), "max": max(step_ms)},
-        "phase_ms": {"sort": statistics.mean(s.sample_ms for s in stats), "lookup": mean_lookup_ms},
-        "roofline": {"bound": "hbm", "kernel": "k_lookup_staged" if a.search == "S" and a.sort == "material_energy" else "k_lookup", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic,
-                     "bytes_per_lookup_alg": bpl, "peak_source": peak_src,
-                     "note": "achieved = SURVEY.md §8d random-gather bytes (E[nuclides] x 96 B per lookup) / "
-                             "k_lookup event time.  The (material, energy) sort makes warps share grid "
-                             "points, so DRAM traffic (`traffic`, ncu) is far below the algorithmic bytes "
-                             "and frac can exceed 1; the kernel is latency-bound (DESIGN.md §7)"},
+        "phase_ms": {"sort": main["sort_ms"], "lookup": main["lookup_ms"]},
+        "roofline": main["roofline"],
+        "verification": {"hash": main["hash"], "lookups": main["lookups"], "pairs": main["pairs"],
+                         "golden_match": main["golden_match"], "hash_consistent": main["hash_consistent"],
+                         "golden": "tests/golden/hashes.json (CPU oracle, every rank's range)"},
+        "north_star": north,
+        "workloads": workloads,
         "ab": ab,
-        "verification": {"hash": h, "lookups": nl, "pairs": npairs},
         "gpu_launches": int(sum(s.launches for s in stats)),
         "e2e": e2e,
+        "clocks": clocks,
     }
-    line["clocks"] = clk.summary()
-    if rec and rec.get("warp_inst_per_launch") and line["clocks"].get("sm_mhz"):
-        sms = torch.cuda.get_device_properties(dev).multi_processor_count
-        ips = rec["warp_inst_per_launch"] / (mean_lookup_ms / 1e3)
-        peak_ips = sms * 4 * line["clocks"]["sm_mhz"] * 1e6  # 4 schedulers x 1 warp-instruction/clk
-        line["roofline"]["issue"] = {"achieved_warp_inst_per_s": ips, "peak": peak_ips, "frac": ips / peak_ips,
-                                     "source": "ncu smsp__inst_executed.sum per launch (profiles/) / live event time"}
-        if rec.get("lsu_wavefronts_per_launch"):
-            # the unit that binds the staged kernel: one L1/shared-memory
-            # data-pipe wavefront per SM per clock
-            wps = rec["lsu_wavefronts_per_launch"] / (mean_lookup_ms / 1e3)
-            peak_wps = sms * line["clocks"]["sm_mhz"] * 1e6
-            line["roofline"]["l1_data_pipe"] = {
-                "achieved_wavefronts_per_s": wps, "peak": peak_wps, "frac": wps / peak_wps,
-                "ncu_pct_of_peak": rec.get("lsu_wavefronts_pct_of_peak"),
-                "source": "ncu shared + global + local LSU wavefronts per launch (profiles/) / live event time"}
-    try:  # SURVEY.md §8d's measured random-gather roofline (tools/l2_gather.cu on this pool's B200)
-        with open(os.path.join(ROOT, "profiles", "l2_gather.json")) as f:
-            lg = json.load(f)
-        key = {"small": "small_points_37MB", "large": "large_points_193MB", "large-U": "large_points_193MB",
-               "XL": "xl_points_4.07GB"}.get(w.name)
-        if key and lg["gathers"].get(key):
-            gp = lg["gathers"][key]["GBps_useful"]
-            line["roofline"]["random_gather"] = {
-                "peak": gp, "unit": "GB/s", "frac": achieved / gp, "buffer": key,
-                "source": "profiles/l2_gather.json: random 96 B record gathers over a buffer the size of this "
-                          "workload's point records (L2-resident for small); frac > 1 = the sort turns the "
-                          "random gather into shared accesses"}
-    except Exception:
-        pass
-    if not a.no_cpu_baseline and R.world == 1:
-        cb = cpu_baseline(w, count, a.cpu_seconds)
-        # parity of the bench's own configuration on the oracle's sample range
-        gs = g.lookup_range(0, cb["_n"], LOOKUP_SEED, None, search=a.search, sort=a.sort)
-        line["verification"]["oracle_sample_hash_match"] = bool(gs.hash == cb["_hash"])
+    if cb:
+        line["verification"]["oracle_sample_hash_match"] = cb["_match"]
         line["cpu_baseline"] = {k: v for k, v in cb.items() if not k.startswith("_")}
     print(json.dumps(line), flush=True)
-    g.close()
     driver.finalize()
+
+
+# ------------------------------------------------------------------ launcher
+def _free_port() -> int:
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def relaunch(a) -> int:
+    """--gpus N without a torchrun environment: run this script under torch.distributed.run,
+    one process per GPU, and return its exit code (rank 0 prints the JSON line)."""
+    env = dict(os.environ)
+    if (env.get("XS_DIST_BACKEND") or "nccl") == "nccl":
+        env.setdefault("NCCL_DEBUG", "INFO")          # the communicator's nranks in the log
+        env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd, env=env)
 
 
 def main():
@@ -400,9 +584,12 @@ def main():
     w = WORKLOADS[a.workload]
     if a.impl == "reference":
         run_reference(a, w)
-    else:
-        run_ours(a, w)
+        return 0
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch(a)
+    run_ours(a, w)
+    return 0
 
 
 if __name__ == "__main__":
-    main()
+    sys.exit(main())

@@ -293,8 +293,9 @@ void build_grid(Grid &g)
         cudaFree(tmp);
         tmp = nullptr;
 
-        // ---- separator tree over every nuclide row (XS_SEARCH_W)
-        {
+        // ---- separator tree over every nuclide row (XS_SEARCH_W; only the nuclide-grid
+        // kernels read it: on XL's hash grid it would be ~0.24 GB never used)
+        if (g.grid_type == XS_NUCLIDE) {
             int64_t R = n;
             g.t_levels = 0;
             int64_t nodes = 1, off = 0;
@@ -320,8 +321,9 @@ void build_grid(Grid &g)
                 XS_CUDA_TRY(cudaGetLastError());
             }
         }
-        // ---- bin bounds over every nuclide row (XS_SEARCH_H): 2^k >= n bins, capped
-        {
+        // ---- bin bounds over every nuclide row (XS_SEARCH_H / S on the nuclide grid only;
+        // the unionized grid bounds its U search with ubnd, the hash grid uses H): 2^k >= n bins
+        if (g.grid_type == XS_NUCLIDE) {
             int b_log2 = 1;
             while ((int64_t(1) << b_log2) < g.n && b_log2 < 20)
                 b_log2++;

@@ -50,6 +50,9 @@ constexpr int kStageCap = XS_STAGE_CAP; // intervals per warp
 #endif
 constexpr int kSortMinNucs = XS_S_SORT_MIN; // sort a warp's lookups when their material has >= this many nuclides
 constexpr int kIvDoubles = 14;
+// stage_interval reads points k and k+1 of a 48 B point-record row; the XS_IV build points
+// NucRef.pts at 96 B interval records instead, which this kernel does not stage
+static_assert(!kIv, "XS_SEARCH_S stages 48 B point records: build without -DXS_IV");
 struct alignas(16) StageMeta {
     double conc;
     int32_t lo;     // L(q_min) of the nuclide

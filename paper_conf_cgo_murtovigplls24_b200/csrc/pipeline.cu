@@ -142,8 +142,8 @@ constexpr int64_t kChunkSorted = int64_t(1) << 28;
 constexpr int64_t kChunkSplit = int64_t(1) << 25;  // pair buffer <= 33.5M x 321 x 4 B
 constexpr int64_t kChunkHost = int64_t(1) << 22;   // staging for host outputs (x2 buffers)
 
-void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
-                 int32_t *out_idx, xs_stats *st)
+static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o,
+                             double *out_macro, int32_t *out_idx, xs_stats *st)
 {
     XS_CHECK_ARG(o.search >= 0 && o.search < XS_SEARCH_COUNT, "opts.search out of range");
     XS_CHECK_ARG(o.sort >= XS_SORT_NONE && o.sort <= XS_SORT_HISTORY, "opts.sort out of range");
@@ -326,6 +326,24 @@ void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_
         st->search_ms = search_ms;
         st->copy_ms = copy_ms;
         st->launches = launches;
+    }
+}
+
+// xs.h promises synchronous calls: if a launch or copy fails partway through the chunk loop,
+// wait for whatever was already queued on the call's stream and the copy stream (ignoring
+// their errors) before the error reaches the caller, so no kernel or D2H copy can still write
+// into the caller's buffers after the call returned
+void run_lookups(Grid &g, int64_t first, int64_t count, uint64_t seed, const xs_opts &o, double *out_macro,
+                 int32_t *out_idx, xs_stats *st)
+{
+    try {
+        run_lookups_impl(g, first, count, seed, o, out_macro, out_idx, st);
+    } catch (...) {
+        cudaStreamSynchronize((cudaStream_t)o.stream);
+        if (g.copy_stream)
+            cudaStreamSynchronize(g.copy_stream);
+        cudaGetLastError();
+        throw;
     }
 }
 

@@ -28,8 +28,16 @@ class Rank:
         return self.world > 1
 
 
+def local_device(local: int) -> int:
+    """The GPU of local rank `local`: one per GPU; with more ranks than visible GPUs (a gloo
+    test of the N > 1 path on a 1-GPU box) ranks share them round-robin."""
+    n = torch.cuda.device_count()
+    return local % n if n > 0 else 0
+
+
 def init(backend: str | None = None) -> Rank:
-    """Join the process group torchrun describes (RANK/WORLD_SIZE/LOCAL_RANK/MASTER_*)."""
+    """Join the process group torchrun describes (RANK/WORLD_SIZE/LOCAL_RANK/MASTER_*).
+    backend: "nccl" (default with CUDA: NVLink / NVSwitch on the B200 node) or "gloo"."""
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -37,13 +45,22 @@ def init(backend: str | None = None) -> Rank:
         if backend is None:
             backend = "nccl" if torch.cuda.is_available() else "gloo"
         if backend == "nccl":
+            if torch.cuda.device_count() < world:
+                raise RuntimeError(f"nccl needs one GPU per rank: {world} ranks, "
+                                   f"{torch.cuda.device_count()} GPUs (XS_DIST_BACKEND=gloo shares them)")
             torch.cuda.set_device(local)
             dist.init_process_group(backend, device_id=torch.device("cuda", local))
         else:
+            if torch.cuda.is_available():
+                torch.cuda.set_device(local_device(local))
             dist.init_process_group(backend)
     elif torch.cuda.is_available():
-        torch.cuda.set_device(local)
+        torch.cuda.set_device(local_device(local))
     return Rank(rank, world, local)
+
+
+def backend_name() -> str:
+    return dist.get_backend() if dist.is_initialized() else "none (1 process)"
 
 
 def shard(total: int, rank: int, world: int) -> tuple[int, int]:
@@ -90,6 +107,22 @@ def replicas_identical(checksum: int, device=None) -> bool:
     dist.all_reduce(lo, op=dist.ReduceOp.MIN)
     dist.all_reduce(hi, op=dist.ReduceOp.MAX)
     return int(lo.item()) == int(hi.item())
+
+
+def sum_over_ranks(x: int, device=None) -> int:
+    if not dist.is_initialized() or dist.get_world_size() == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.int64, device=_device(device))
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return int(t.item())
+
+
+def min_over_ranks(x: int, device=None) -> int:
+    if not dist.is_initialized() or dist.get_world_size() == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.int64, device=_device(device))
+    dist.all_reduce(t, op=dist.ReduceOp.MIN)
+    return int(t.item())
 
 
 def max_over_ranks(x: float, device=None) -> float:

@@ -20,8 +20,9 @@ class Workload:
     n_nuclides: int
     n_gridpoints: int
     grid_type: int
-    lookups: int          # per GPU at N=1 (bench weak-scales this per rank)
+    lookups: int          # strong scaling: the job's total; weak scaling: per rank
     note: str
+    scaling: str = "strong"  # bench.py default (SURVEY.md §8e partitions a fixed total)
 
     @property
     def n_points(self) -> int:
@@ -38,7 +39,8 @@ WORKLOADS = {
     # configs[3]: large, unionized (energy-index) grid
     "large-U": Workload("large-U", 355, 11303, UNIONIZED, 100_000_000, "configs[3]"),
     # configs[4]: XL, hash grid with 10,000 bins; 1e9 lookups over 8 GPUs
-    "XL": Workload("XL", 355, 238847, HASH, 1_000_000_000 // 8, "configs[4] (per-GPU share)"),
+    # weak: every rank owns 125M lookups, so N = 8 is exactly the 1B-lookup configuration
+    "XL": Workload("XL", 355, 238847, HASH, 1_000_000_000 // 8, "configs[4] (per-GPU share)", "weak"),
 }
 
 # Mean nuclides per lookup under pick_mat's effective distribution (SURVEY.md §8
