@@ -15,7 +15,7 @@ BUILD = os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 SOURCES = ["api.cu", "grid.cu", "sort.cu", "lookup_fused.cu", "lookup_staged.cu", "lookup_split.cu", "pipeline.cu", "bezier.cu"]
-HEADERS = ["rng.cuh", "search.cuh", "xs_internal.cuh", "lookup_common.cuh"]
+HEADERS = ["rng.cuh", "search.cuh", "search_uu.cuh", "xs_internal.cuh", "lookup_common.cuh"]
 FLAGS = [
     "-O3", "-std=c++17",
     "-gencode", "arch=compute_100a,code=sm_100a",

@@ -103,19 +103,3 @@ def test_product_never_imports_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 text = open(os.path.join(dirpath, f)).read()
                 assert "oracle" not in re.sub(r"#.*|//.*", "", text).lower().replace("oracle/", ""), f
-
-
-def test_sass_shapes_of_search_variants(xs):
-    """Listing 4 vs Listing 5 in SASS: the merged search is select-based (SEL, no branch in
-    the body but the back edge); the unmerged u=2 search has the true-true path guard
-    `length >= 4` (ISETP.GE.U32 ... 0x4) and the `length >> 2` update (SHF.R.U32.HI ... 0x2)."""
-    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", "-fun",
-                           "_ZN2xs15k_search_pointsILi1ELi2EEEvNS_8GridViewElPKdPKiPi", LIB],
-                          capture_output=True, text=True).stdout
-    assert re.search(r"ISETP\.GE\.U32\.AND P\d, PT, R\d+, 0x4", sass)
-    assert re.search(r"SHF\.R\.U32\.HI R\d+, RZ, 0x2, R\d+", sass)
-    merged = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", "-fun",
-                             "_ZN2xs15k_search_pointsILi1ELi0EEEvNS_8GridViewElPKdPKiPi", LIB],
-                            capture_output=True, text=True).stdout
-    assert merged.count("SEL ") >= 2
-    assert merged.count("DSETP") == 1  # one probe per iteration, no unrolled copies
