@@ -154,10 +154,14 @@ def fp64_peak_tflops(sms: int):
 
 
 def libxs_sha() -> str:
+    """The build identity of libxs.so (build.py source_digest: sources + flags)."""
     try:
-        from paper_conf_cgo_murtovigplls24_b200 import _xs
-        with open(_xs.LIB_PATH, "rb") as f:
-            return hashlib.sha256(f.read()).hexdigest()[:16]
+        import importlib.util
+        spec = importlib.util.spec_from_file_location(
+            "_xs_build", os.path.join(ROOT, "paper_conf_cgo_murtovigplls24_b200", "build.py"))
+        b = importlib.util.module_from_spec(spec)
+        spec.loader.exec_module(b)
+        return b.source_digest()
     except Exception:
         return ""
 

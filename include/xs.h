@@ -51,8 +51,8 @@ enum { XS_OK = 0, XS_EINVAL = -1, XS_ENOMEM = -2, XS_ECUDA = -3, XS_EDUP = -4 };
  * the paper measures (Listings 4 and 5).                       */
 enum {
     XS_SEARCH_M = 0,  /* merged: Listing 3 as written (select-based, Listing 4 shape)  */
-    XS_SEARCH_U1 = 1, /* unmerged: each branch carries its own length update        */
-    XS_SEARCH_U2 = 2, /* unmerged + unrolled x2 (Listing 5: TT path has no subtract)  */
+    XS_SEARCH_U1 = 1, /* unmerged: each branch its own length update + loop test    */
+    XS_SEARCH_U2 = 2, /* unmerged + unrolled x2, 4 paths with own back edges (L. 5) */
     XS_SEARCH_U4 = 3, /* unmerged + unrolled x4 (2^4 leaf paths)        */
     XS_SEARCH_U8 = 4, /* unmerged + unrolled x8 (2^8 leaf paths)                      */
     XS_SEARCH_B = 5,  /* branchless select form of the unmerged update               */

@@ -27,6 +27,21 @@ FLAGS = [
 ]
 
 
+def source_digest() -> str:
+    """sha256 (16 hex) over every source, header and flag that goes into libxs.so: the build
+    identity profiles/ncu_traffic.json records are keyed by (deterministic, unlike the binary's
+    own bytes across rebuilds)."""
+    import hashlib
+    h = hashlib.sha256()
+    for f in sorted(SOURCES + HEADERS):
+        with open(os.path.join(CSRC, f), "rb") as fh:
+            h.update(f.encode() + b"\0" + fh.read())
+    with open(os.path.join(INCLUDE, "xs.h"), "rb") as fh:
+        h.update(fh.read())
+    h.update(" ".join(f for f in FLAGS if not f.startswith("/")).encode())
+    return h.hexdigest()[:16]
+
+
 def _stale() -> bool:
     if not os.path.exists(LIB):
         return True

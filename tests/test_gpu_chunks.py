@@ -65,7 +65,7 @@ print("WINDOWS OK")
 """ % ROOT
 
 
-@pytest.mark.parametrize("windows", [2, 7, 39])
+@pytest.mark.parametrize("windows", [1, 2, 7, 39])
 def test_scatter_windows_match_oracle(windows):
     """the windowed scatter (one launch per window of buckets) with the window count forced
     (XS_TEST_SCATTER_WINDOWS): every bucket is written by exactly one window"""

@@ -35,6 +35,18 @@ for st in "$@"; do
                 timeout 1500 ncu --set full --clock-control none --import-source on \
                   -k regex:"k_lookup|k_bucket" --launch-skip 12 --launch-count 6 -f -o $OUT/${TAG}_${S}_${W} \
                   python tools/ncu_target.py $W $S $SORT 4 > $OUT/${TAG}_ncu_${W}_${S}.log 2>&1 ;;
+    ncuk:*)     IFS=: read -r _ W S SORT <<< "$st"; SORT=${SORT:-material_energy}
+                timeout 1500 ncu --set full --clock-control none --import-source on \
+                  -k regex:k_lookup --launch-skip 1 --launch-count 1 -f -o $OUT/${TAG}_${S}_${W}_${SORT} \
+                  python tools/ncu_target.py $W $S $SORT 2 > $OUT/${TAG}_ncuk_${W}_${S}_${SORT}.log 2>&1 ;;
+    ncusort:*)  W=${st#ncusort:}
+                timeout 1500 ncu --set full --clock-control none --import-source on \
+                  -k regex:k_bucket --launch-skip 24 --launch-count 24 -f -o $OUT/${TAG}_sort_${W} \
+                  python tools/ncu_target.py $W S material_energy 4 > $OUT/${TAG}_ncusort_${W}.log 2>&1 ;;
+    abncu:*)    W=${st#abncu:}
+                timeout 1800 ncu --metrics smsp__thread_inst_executed_per_inst_executed.ratio,smsp__inst_executed.sum,sm__inst_executed.avg.per_cycle_active,smsp__sass_average_branch_targets_threads_uniform.pct,smsp__warp_issue_stalled_no_instruction_per_warp_active.pct,l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum,l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum,lts__t_sector_hit_rate.pct,dram__bytes_read.sum,gpu__time_duration.sum,sass__inst_executed_per_opcode \
+                  --print-metric-instances values --csv -k regex:k_lookup --log-file $OUT/${TAG}_abncu_${W}.csv \
+                  python tools/ab_sweep.py --workload $W --ncu --lookups 4000000 > $OUT/${TAG}_abncu_${W}.log 2>&1 ;;
     kt:*)       W=${st#kt:}; timeout 600 python tools/kernel_times.py $W S > $OUT/${TAG}_kt_${W}.log 2>&1 ;;
     probes)     for t in lds_probe fp64_peak l2_gather; do
                   [ -x tools/$t ] || nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o tools/$t tools/$t.cu
