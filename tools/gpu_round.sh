@@ -45,7 +45,7 @@ for st in "$@"; do
                   python tools/ncu_target.py $W S material_energy 4 > $OUT/${TAG}_ncusort_${W}.log 2>&1 ;;
     abncu:*)    W=${st#abncu:}
                 timeout 1800 ncu --metrics smsp__thread_inst_executed_per_inst_executed.ratio,smsp__inst_executed.sum,sm__inst_executed.avg.per_cycle_active,smsp__sass_average_branch_targets_threads_uniform.pct,smsp__warp_issue_stalled_no_instruction_per_warp_active.pct,l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum,l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum,lts__t_sector_hit_rate.pct,dram__bytes_read.sum,gpu__time_duration.sum,sass__inst_executed_per_opcode \
-                  --print-metric-instances values --csv -k regex:k_lookup --log-file $OUT/${TAG}_abncu_${W}.csv \
+                  --print-metric-instances details --csv -k regex:k_lookup --log-file $OUT/${TAG}_abncu_${W}.csv \
                   python tools/ab_sweep.py --workload $W --ncu --lookups 4000000 > $OUT/${TAG}_abncu_${W}.log 2>&1 ;;
     kt:*)       W=${st#kt:}; timeout 600 python tools/kernel_times.py $W S > $OUT/${TAG}_kt_${W}.log 2>&1 ;;
     probes)     for t in lds_probe fp64_peak l2_gather; do
