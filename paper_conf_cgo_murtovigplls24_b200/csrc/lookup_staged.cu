@@ -6,6 +6,7 @@
 // and every nuclide of the material is resolved through a window of interval records staged
 // in shared memory.
 #include <algorithm>
+#include <cstddef>
 
 #include "lookup_common.cuh"
 
@@ -53,11 +54,13 @@ constexpr int kIvDoubles = 14;
 // stage_interval reads points k and k+1 of a 48 B point-record row; the XS_IV build points
 // NucRef.pts at 96 B interval records instead, which this kernel does not stage
 static_assert(!kIv, "XS_SEARCH_S stages 48 B point records: build without -DXS_IV");
+
 struct alignas(16) StageMeta {
     double conc;
     int32_t lo;     // L(q_min) of the nuclide
     int32_t offcnt; // (first staged interval << 16) | intervals, or -1: not staged
 };
+static_assert(sizeof(StageMeta) == 16 && offsetof(StageMeta, offcnt) == 12, "the hot loop reads offcnt at byte 12");
 constexpr int kStageWarpBytes = kStageCap * kIvDoubles * 8 + kStageCap * 8 + 32 * (int)sizeof(StageMeta) +
                                 32 * 8 + 32 * 4 + ((kStageCap + 15) / 16) * 16;
 
@@ -70,7 +73,12 @@ struct WarpStage {
     const double **pts;  // [32] point row of the nuclide
     int *cnt;            // [32] intervals of the nuclide's window
     uint8_t *owner;      // [kStageCap]
+    // the hot loop's view: byte offsets into st_smem (32-bit shared addressing; generic 64-bit
+    // pointers were rematerialised from SR_TID / SR_CgaCtaId for every nuclide)
+    int orec, oeh, ometa;
 };
+
+extern __shared__ __align__(16) unsigned char st_smem[]; // k_lookup_staged's dynamic shared memory
 
 __device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
 {
@@ -82,6 +90,12 @@ __device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
     w.pts = reinterpret_cast<const double **>(w.meta + 32);
     w.cnt = reinterpret_cast<int *>(w.pts + 32);
     w.owner = reinterpret_cast<uint8_t *>(w.cnt + 32);
+    // opaque: kept in registers, not re-derived from SR_TID.X (a long-latency S2R) per nuclide
+    int o = (int)(threadIdx.x >> 5) * kStageWarpBytes;
+    asm("mov.b32 %0, %0;" : "+r"(o));
+    w.orec = o;
+    w.oeh = o + kStageCap * kIvDoubles * 8;
+    w.ometa = w.oeh + kStageCap * 8;
     return w;
 }
 
@@ -208,15 +222,15 @@ __device__ __forceinline__ void warp_sort(uint64_t (&k)[kLpl], uint32_t (&v)[kLp
 // path.  `col` is the nuclide's column in out_idx.
 template <int GRID, bool OUTS, bool ALL = false>
 __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx, int col, const int offcnt,
-                                                const StageMeta *mp, const double *eh_all, const double *rec_all,
+                                                const StageMeta *mp, int oeh, int orec,
                                                 const bool (&mine)[kLpl], const double (&q)[kLpl],
                                                 const uint32_t (&r)[kLpl], int32_t *__restrict__ out_idx,
                                                 Acc (&A)[kLpl])
 {
     if (offcnt >= 0) {
         const int off_w = offcnt >> 16, cnt_w = offcnt & 0xFFFF;
-        const double *eh = eh_all + off_w;
-        const double *R = rec_all + off_w * kIvDoubles;
+        const double *eh = reinterpret_cast<const double *>(st_smem + oeh) + off_w;
+        const double *R = reinterpret_cast<const double *>(st_smem + orec) + off_w * kIvDoubles;
         // branch-free over the lane's lookups, so their FP64 chains interleave: a lookup
         // that is not `mine` accumulates with concentration +0, fma(micro, +0, acc) == acc
         // exactly (micro is finite and acc is never -0)
@@ -355,21 +369,23 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
             __syncwarp();
             // ascending nuclide order (R8); the next nuclide's window descriptor is read one
             // nuclide ahead (the record load depends on it)
-            int oc = ws.meta[b0].offcnt;
+            // the offcnt words of the pass's nuclides: StageMeta is 16 B, offcnt at byte 12
+            const int *ocp = reinterpret_cast<const int *>(st_smem + ws.ometa + 12);
+            int oc = ocp[4 * b0];
 #if XS_S_ALL
             if (all_mine) { // every lookup of the warp is this material's (the sorted norm): no selects
                 for (int jj = b0; jj < b1; jj++) {
-                    const int oc_next = jj + 1 < b1 ? ws.meta[jj + 1].offcnt : 0;
-                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.eh, ws.rec,
+                    const int oc_next = jj + 1 < b1 ? ocp[4 * (jj + 1)] : 0;
+                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.oeh, ws.orec,
                                                       mine, q, r, out_idx, A);
                     oc = oc_next;
                 }
             } else
 #endif
                 for (int jj = b0; jj < b1; jj++) {
-                    const int oc_next = jj + 1 < b1 ? ws.meta[jj + 1].offcnt : 0;
-                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.eh, ws.rec, mine, q,
-                                                r, out_idx, A);
+                    const int oc_next = jj + 1 < b1 ? ocp[4 * (jj + 1)] : 0;
+                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.oeh, ws.orec, mine,
+                                                q, r, out_idx, A);
                     oc = oc_next;
                 }
             b0 = b1;
@@ -454,7 +470,6 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
     pdl_wait(); // the sort's outputs (and the work counter it zeroed) are complete
     double *__restrict__ out = OUTS ? out_ : nullptr;
     int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
-    extern __shared__ __align__(16) unsigned char st_smem[];
     __shared__ uint32_t s_mb[kMaterials + 1];
     if (threadIdx.x <= kMaterials)
         s_mb[threadIdx.x] = __ldg(so.mb_dev + threadIdx.x);
