@@ -29,6 +29,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_WSORT
 #define XS_S_WSORT 0
 #endif
+#ifndef XS_S_CNT2
+#define XS_S_CNT2 1
+#endif
 #ifndef XS_S_FASTMASK
 #define XS_S_FASTMASK 1
 #endif
@@ -254,8 +257,15 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             const double e3 = cnt_w > 3 ? eh[2] : inf;
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
-                // E[lo + k] = eh[k - 1], k = 1..cnt-1
+                // E[lo + k] = eh[k - 1], k = 1..cnt-1 ascending: c = #{e_k <= q} by two
+                // compares (e2 first, then e3 or e1) instead of three
+#if XS_S_CNT2
+                const bool p2 = e2 <= q[l];
+                const double e = p2 ? e3 : e1;
+                const int c = (p2 ? 2 : 0) + (e <= q[l] ? 1 : 0);
+#else
                 const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
+#endif
                 const IvRec v = load_rec(R + c * kIvDoubles);
                 accumulate_interval(v, q[l], (ALL || mine[l]) ? v.e.y : 0.0, A[l]);
                 if constexpr (OUTS) {
