@@ -29,6 +29,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_WSORT
 #define XS_S_WSORT 0
 #endif
+#ifndef XS_S_STAGE2
+#define XS_S_STAGE2 1
+#endif
 #ifndef XS_S_CNT2
 #define XS_S_CNT2 1
 #endif
@@ -52,6 +55,7 @@ constexpr int kLpl = XS_S_LPL; // lookups per lane per iteration: they share the
 #define XS_STAGE_CAP 48
 #endif
 constexpr int kStageCap = XS_STAGE_CAP; // intervals per warp
+static_assert(!XS_S_STAGE2 || kStageCap <= 64, "the two-interval staging covers at most 64 intervals per pass");
 #ifndef XS_S_SORT_MIN
 #define XS_S_SORT_MIN 64
 #endif
@@ -141,12 +145,19 @@ __device__ __forceinline__ void accumulate_interval(const IvRec &v, double q, do
 }
 
 // interval record k of a point row (points k and k+1) into shared memory
-__device__ __forceinline__ void stage_interval(const double *__restrict__ pts, int k, double *dst, double *eh,
-                                               double conc)
+struct RawIv { // points k and k+1 of a 48 B point-record row
+    double2 a0, a1, a2, b0, b1, b2;
+};
+
+__device__ __forceinline__ RawIv load_raw(const double *__restrict__ pts, int k)
 {
     const double2 *p = reinterpret_cast<const double2 *>(pts) + (size_t)(uint32_t)k * 3;
-    const double2 a0 = __ldg(p), a1 = __ldg(p + 1), a2 = __ldg(p + 2);
-    const double2 b0 = __ldg(p + 3), b1 = __ldg(p + 4), b2 = __ldg(p + 5);
+    return RawIv{__ldg(p), __ldg(p + 1), __ldg(p + 2), __ldg(p + 3), __ldg(p + 4), __ldg(p + 5)};
+}
+
+__device__ __forceinline__ void store_interval(const RawIv &v, double *dst, double *eh, double conc)
+{
+    const double2 a0 = v.a0, a1 = v.a1, a2 = v.a2, b0 = v.b0, b1 = v.b1, b2 = v.b2;
     const double d = __dsub_rn(b0.x, a0.x);
     double2 *o = reinterpret_cast<double2 *>(dst) + 1;
     o[-1] = make_double2(b0.x, conc); // the nuclide's concentration rides in the pad slot
@@ -157,6 +168,12 @@ __device__ __forceinline__ void stage_interval(const double *__restrict__ pts, i
     o[4] = make_double2(b2.x, __dsub_rn(b2.x, a2.x));
     o[5] = make_double2(b2.y, __dsub_rn(b2.y, a2.y));
     *eh = b0.x;
+}
+
+__device__ __forceinline__ void stage_interval(const double *__restrict__ pts, int k, double *dst, double *eh,
+                                               double conc)
+{
+    store_interval(load_raw(pts, k), dst, eh, conc);
 }
 
 // c = #{k in 1..cnt-1 : E[lo + k] <= q} (E[lo + k] = eh[k - 1]), i.e. L(q) - lo: short
@@ -374,11 +391,32 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
             }
             __syncwarp();
             // interval i of the pass is staged by lane i % 32: owner nuclide j, its k-th interval
+#if XS_S_STAGE2
+            // each lane stages intervals lane and lane + 32 (T <= kStageCap <= 64): the second
+            // interval's six loads are issued with the first's, so a pass waits for one
+            // memory latency instead of two
+            {
+                const int i1 = lane + 32;
+                const bool h0 = lane < T, h1 = i1 < T;
+                const int j0 = h0 ? ws.owner[lane] : 0, j1 = h1 ? ws.owner[i1] : 0;
+                const StageMeta m0 = ws.meta[j0], m1 = ws.meta[j1];
+                RawIv v0{}, v1{};
+                if (h0)
+                    v0 = load_raw(ws.pts[j0], m0.lo + (lane - (m0.offcnt >> 16)));
+                if (h1)
+                    v1 = load_raw(ws.pts[j1], m1.lo + (i1 - (m1.offcnt >> 16)));
+                if (h0)
+                    store_interval(v0, ws.rec + lane * kIvDoubles, ws.eh + lane, m0.conc);
+                if (h1)
+                    store_interval(v1, ws.rec + i1 * kIvDoubles, ws.eh + i1, m1.conc);
+            }
+#else
             for (int i = lane; i < T; i += 32) {
                 const int j = ws.owner[i];
                 const StageMeta mj = ws.meta[j];
                 stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i, mj.conc);
             }
+#endif
             __syncwarp();
             // ascending nuclide order (R8); the next nuclide's window descriptor is read one
             // nuclide ahead (the record load depends on it)

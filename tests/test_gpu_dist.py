@@ -112,3 +112,20 @@ def test_bench_one_rank_golden_and_contract():
     assert d["workloads"]["small"]["golden_match"] is True
     assert d["workloads"]["small"]["roofline"]["frac"] <= 1.0
     assert d["gpu_launches"] > 0
+
+
+def test_bench_nccl_all_gpus():
+    """The production path: one rank per GPU over NCCL (NVLink / NVSwitch), launched by
+    bench.py itself -- runs only where more than one GPU is visible (an 8-GPU node)."""
+    if not torch.cuda.is_available() or torch.cuda.device_count() < 2:
+        pytest.skip("needs >= 2 GPUs")
+    n = min(torch.cuda.device_count(), 8)
+    env = {k: v for k, v in os.environ.items() if k != "XS_DIST_BACKEND"}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", str(n), "--workload", "tiny",
+                        "--steps", "3", "--warmup", "3", "--ab", "", "--workloads", "", "--no-e2e",
+                        "--no-cpu-baseline"], capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    gd = GOLDEN["tiny"]
+    assert d["n_gpus"] == n and d["path"]["backend"] == "nccl"
+    assert d["verification"]["hash"] == gd["hash_total"] and d["verification"]["golden_match"] is True
