@@ -82,6 +82,28 @@ __global__ void k_fill_points(uint64_t seed, int64_t N, int32_t n, double *__res
     }
 }
 
+// the staged kernel's interval records (XS_S_TMA): ivs[i] for interval L = i mod (n-1) of
+// nuclide i / (n-1), 14 doubles, rounded exactly as lookup_staged.cu's stage_interval rounds
+// them (so results stay bit-identical); slot 1 (the concentration there) is 0 here
+__global__ void k_ivs_build(int64_t NI, int32_t n, const double *__restrict__ pts, double *__restrict__ ivs)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < NI; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t nuc = i / (n - 1), L = i - nuc * (n - 1);
+        const double *lo = pts + (nuc * n + L) * 6, *hi = lo + 6;
+        double *o = ivs + i * 14;
+        const double d = __dsub_rn(hi[0], lo[0]);
+        o[0] = hi[0];
+        o[1] = 0.0;
+        o[2] = d;
+        o[3] = __drcp_rn(d);
+#pragma unroll
+        for (int c = 0; c < 5; c++) {
+            o[4 + 2 * c] = hi[1 + c];
+            o[5 + 2 * c] = __dsub_rn(hi[1 + c], lo[1 + c]);
+        }
+    }
+}
+
 // interval records (XS_IV): iv[i] for interval L = i mod (n-1) of nuclide i / (n-1)
 __global__ void k_iv_build(int64_t NI, int32_t n, const double *__restrict__ pts, double *__restrict__ iv)
 {
@@ -286,6 +308,12 @@ void build_grid(Grid &g)
             k_iv_build<<<grid_blocks(NI, tpb), tpb>>>(NI, n, g.pts, g.iv);
             XS_CUDA_TRY(cudaGetLastError());
         }
+        if (kTmaStage && g.grid_type == XS_HASH) { // the staged kernel's bulk-copied records (hash grid)
+            const int64_t NI = g.n_nuc * (n - 1);
+            g.ivs = dalloc<double>(g, NI * 14);
+            k_ivs_build<<<grid_blocks(NI, tpb), tpb>>>(NI, n, g.pts, g.ivs);
+            XS_CUDA_TRY(cudaGetLastError());
+        }
         int dup_h = 0;
         XS_CUDA_TRY(cudaMemcpy(&dup_h, dup, sizeof(int), cudaMemcpyDeviceToHost));
         if (dup_h)
@@ -422,6 +450,7 @@ void free_grid(Grid &g)
     cudaFree(g.E);
     cudaFree(g.pts);
     cudaFree(g.iv);
+    cudaFree(g.ivs);
     cudaFree(g.tkeys);
     cudaFree(g.bnd);
     cudaFree(g.ubnd);
@@ -493,6 +522,7 @@ GridView make_view(const Grid &g)
     v.E = g.E;
     v.pts = g.pts;
     v.iv = g.iv;
+    v.ivs = g.ivs;
     v.U = g.U;
     v.IDX = g.IDX;
     v.H = g.H;

@@ -12,7 +12,10 @@
 
 namespace xs {
 
-constexpr int kStTpb = 256;
+#ifndef XS_S_TPB
+#define XS_S_TPB 256
+#endif
+constexpr int kStTpb = XS_S_TPB;
 #ifndef XS_S_MIN_BLOCKS
 #define XS_S_MIN_BLOCKS 2
 #endif
@@ -61,9 +64,16 @@ static_assert(!XS_S_STAGE2 || kStageCap <= 64, "the two-interval staging covers 
 #endif
 constexpr int kSortMinNucs = XS_S_SORT_MIN; // sort a warp's lookups when their material has >= this many nuclides
 constexpr int kIvDoubles = 14;
+// XS_S_TMA applies to the hash grid (XL): bulk-copied records took XL's lookup kernel from
+// 19.33 to 18.42 ms but the nuclide / unionized ones 2-6% slower (their windows are mostly
+// one interval, staging is cheap there, and the 112 B records double the L2 footprint of 48 B
+// points) -- DESIGN.md §6.8
+template <int GRID> constexpr bool kTma = kTmaStage && GRID == XS_HASH;
+template <int GRID> constexpr int kEhStride = kTma<GRID> ? kIvDoubles : 1; // stride of the upper energies
 // stage_interval reads points k and k+1 of a 48 B point-record row; the XS_IV build points
 // NucRef.pts at 96 B interval records instead, which this kernel does not stage
 static_assert(!kIv, "XS_SEARCH_S stages 48 B point records: build without -DXS_IV");
+static_assert(kIvDoubles * 8 % 16 == 0, "bulk copies move whole 16 B units");
 
 struct alignas(16) StageMeta {
     double conc;
@@ -72,7 +82,7 @@ struct alignas(16) StageMeta {
 };
 static_assert(sizeof(StageMeta) == 16 && offsetof(StageMeta, offcnt) == 12, "the hot loop reads offcnt at byte 12");
 constexpr int kStageWarpBytes = kStageCap * kIvDoubles * 8 + kStageCap * 8 + 32 * (int)sizeof(StageMeta) +
-                                32 * 8 + 32 * 4 + ((kStageCap + 15) / 16) * 16;
+                                32 * 8 + 32 * 4 + ((kStageCap + 15) / 16) * 16 + 16;
 
 // The group's per-nuclide state lives in shared memory, not in registers, while the
 // group is computed (registers decide the occupancy of this kernel).
@@ -83,6 +93,7 @@ struct WarpStage {
     const double **pts;  // [32] point row of the nuclide
     int *cnt;            // [32] intervals of the nuclide's window
     uint8_t *owner;      // [kStageCap]
+    uint64_t *mbar;      // XS_S_TMA: the warp's mbarrier for the bulk copies of a pass
     // the hot loop's view: byte offsets into st_smem (32-bit shared addressing; generic 64-bit
     // pointers were rematerialised from SR_TID / SR_CgaCtaId for every nuclide)
     int orec, oeh, ometa;
@@ -100,6 +111,7 @@ __device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
     w.pts = reinterpret_cast<const double **>(w.meta + 32);
     w.cnt = reinterpret_cast<int *>(w.pts + 32);
     w.owner = reinterpret_cast<uint8_t *>(w.cnt + 32);
+    w.mbar = reinterpret_cast<uint64_t *>(w.owner + ((kStageCap + 15) / 16) * 16);
     // opaque: kept in registers, not re-derived from SR_TID.X (a long-latency S2R) per nuclide
     int o = (int)(threadIdx.x >> 5) * kStageWarpBytes;
     asm("mov.b32 %0, %0;" : "+r"(o));
@@ -107,6 +119,36 @@ __device__ __forceinline__ WarpStage warp_stage(unsigned char *smem)
     w.oeh = o + kStageCap * kIvDoubles * 8;
     w.ometa = w.oeh + kStageCap * 8;
     return w;
+}
+
+// ---- XS_S_TMA: interval records copied by the bulk-copy engine (cp.async.bulk, UBLKCP) ----
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *mb)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(mb)));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *mb, unsigned bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(mb)), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *mb, unsigned phase)
+{
+    asm volatile("{\n\t.reg .pred P;\n"
+                 "XS_WAIT_%=:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+                 "@!P bra XS_WAIT_%=;\n\t}" ::"r"(smem_u32(mb)), "r"(phase) : "memory");
+}
+
+// `bytes` (a multiple of 16) from global `src` to shared `dst` (both 16 B aligned), completing
+// on the mbarrier's transaction count
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *mb)
+{
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(mb)) : "memory");
 }
 
 // f = RN(a / d) from y = RN(1/d): q0 = RN(a y), r = a - d q0 (exact, an FMA), f = RN(q0 + r y).
@@ -179,12 +221,13 @@ __device__ __forceinline__ void stage_interval(const double *__restrict__ pts, i
 // c = #{k in 1..cnt-1 : E[lo + k] <= q} (E[lo + k] = eh[k - 1]), i.e. L(q) - lo: short
 // windows by three compares of values shared by the lane's lookups, longer ones by Listing 1
 // (U1) over eh
+template <int EHS>
 __device__ __forceinline__ int window_count(const double *eh, int cnt, double q)
 {
     int c = 0, len = cnt;
     while (len > 1) {
         const int h = len >> 1;
-        if (eh[c + h - 1] > q) {
+        if (eh[(c + h - 1) * EHS] > q) {
             len = h;
         } else {
             c += h;
@@ -252,8 +295,13 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
 {
     if (offcnt >= 0) {
         const int off_w = offcnt >> 16, cnt_w = offcnt & 0xFFFF;
-        const double *eh = reinterpret_cast<const double *>(st_smem + oeh) + off_w;
         const double *R = reinterpret_cast<const double *>(st_smem + orec) + off_w * kIvDoubles;
+        // upper energies E[lo + k] = eh[(k - 1) kEhStride]: the compact array, or (bulk-copied
+        // records) the records' own first field
+        const double *eh = kTma<GRID> ? R : reinterpret_cast<const double *>(st_smem + oeh) + off_w;
+        // the nuclide's concentration: in the record's pad slot, or (bulk-copied records, which
+        // are shared by every material) from the descriptor
+        const double conc = kTma<GRID> ? mp->conc : 0.0;
         // branch-free over the lane's lookups, so their FP64 chains interleave: a lookup
         // that is not `mine` accumulates with concentration +0, fma(micro, +0, acc) == acc
         // exactly (micro is finite and acc is never -0)
@@ -261,7 +309,7 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
             const IvRec v = load_rec(R);
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
-                accumulate_interval(v, q[l], (ALL || mine[l]) ? v.e.y : 0.0, A[l]);
+                accumulate_interval(v, q[l], (ALL || mine[l]) ? (kTma<GRID> ? conc : v.e.y) : 0.0, A[l]);
                 if constexpr (OUTS) {
                     if (out_idx && mine[l])
                         out_idx[(size_t)r[l] * gv.max_nucs + col] = mp->lo;
@@ -270,8 +318,8 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
         } else if (cnt_w <= 4) { // the upper energies of a short window, shared by the lookups
             const double inf = __longlong_as_double(0x7FF0000000000000ll);
             const double e1 = eh[0];
-            const double e2 = cnt_w > 2 ? eh[1] : inf;
-            const double e3 = cnt_w > 3 ? eh[2] : inf;
+            const double e2 = cnt_w > 2 ? eh[kEhStride<GRID>] : inf;
+            const double e3 = cnt_w > 3 ? eh[2 * kEhStride<GRID>] : inf;
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
                 // E[lo + k] = eh[k - 1], k = 1..cnt-1 ascending: c = #{e_k <= q} by two
@@ -284,7 +332,7 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
                 const int c = (e1 <= q[l] ? 1 : 0) + (e2 <= q[l] ? 1 : 0) + (e3 <= q[l] ? 1 : 0);
 #endif
                 const IvRec v = load_rec(R + c * kIvDoubles);
-                accumulate_interval(v, q[l], (ALL || mine[l]) ? v.e.y : 0.0, A[l]);
+                accumulate_interval(v, q[l], (ALL || mine[l]) ? (kTma<GRID> ? conc : v.e.y) : 0.0, A[l]);
                 if constexpr (OUTS) {
                     if (out_idx && mine[l])
                         out_idx[(size_t)r[l] * gv.max_nucs + col] = mp->lo + c;
@@ -294,9 +342,9 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
                 if (mine[l]) {
-                    const int c = window_count(eh, cnt_w, q[l]);
+                    const int c = window_count<kEhStride<GRID>>(eh, cnt_w, q[l]);
                     const IvRec v = load_rec(R + c * kIvDoubles);
-                    accumulate_interval(v, q[l], v.e.y, A[l]);
+                    accumulate_interval(v, q[l], kTma<GRID> ? conc : v.e.y, A[l]);
                     if constexpr (OUTS) {
                         if (out_idx)
                             out_idx[(size_t)r[l] * gv.max_nucs + col] = mp->lo + c;
@@ -326,7 +374,7 @@ __device__ __forceinline__ void compute_nuclide(const GridView &gv, int ref_idx,
 // The lookups in `mine` (one material: row `roww`, nn nuclides; kLpl per lane) accumulate
 // every nuclide of the material.  All 32 lanes call it (warp collectives inside).
 template <int GRID, bool OUTS>
-__device__ __forceinline__ void staged_material(const GridView &gv, int roww, int nn, const bool (&mine)[kLpl],
+__device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tma_phase, int roww, int nn, const bool (&mine)[kLpl],
                                                 const double (&q)[kLpl], const uint32_t (&r)[kLpl],
                                                 const WarpStage &ws, int32_t *__restrict__ out_idx,
                                                 Acc (&A)[kLpl])
@@ -362,7 +410,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
             const int lo = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_lo, e_lo);
             ws.cnt[lane] = lower_index<GRID, XS_SEARCH_S>(gv, rw, q_hi, e_hi) - lo + 1;
             ws.meta[lane] = StageMeta{rw.conc, lo, 0};
-            ws.pts[lane] = rw.pts;
+            ws.pts[lane] = kTma<GRID> ? gv.ivs + (size_t)rw.nuc * (uint32_t)(gv.n - 1) * kIvDoubles : rw.pts;
         }
         __syncwarp();
         for (int b0 = 0; b0 < ng;) { // passes over the group (warp-uniform)
@@ -391,6 +439,24 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
             }
             __syncwarp();
             // interval i of the pass is staged by lane i % 32: owner nuclide j, its k-th interval
+            if constexpr (kTma<GRID>) {
+                // the pass's windows are contiguous runs of precomputed records (gv.ivs): each
+                // nuclide's lane issues one bulk copy of its window, the warp waits on its
+                // mbarrier for all of them (T intervals x 112 B); no registers, no LSU traffic
+                if (T > 0) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); // prior reads before async writes
+                    if (lane == 0)
+                        mbar_expect_tx(ws.mbar, (unsigned)T * kIvDoubles * 8);
+                    __syncwarp();
+                    if (fits) {
+                        const int off = incl - want;
+                        bulk_g2s(ws.rec + off * kIvDoubles, ws.pts[lane] + (size_t)(uint32_t)ws.meta[lane].lo * kIvDoubles,
+                                 (unsigned)want * kIvDoubles * 8, ws.mbar);
+                    }
+                    mbar_wait(ws.mbar, tma_phase);
+                    tma_phase ^= 1u;
+                }
+            } else {
 #if XS_S_STAGE2
             // each lane stages intervals lane and lane + 32 (T <= kStageCap <= 64): the second
             // interval's six loads are issued with the first's, so a pass waits for one
@@ -417,6 +483,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
                 stage_interval(ws.pts[j], mj.lo + (i - (mj.offcnt >> 16)), ws.rec + i * kIvDoubles, ws.eh + i, mj.conc);
             }
 #endif
+            }
             __syncwarp();
             // ascending nuclide order (R8); the next nuclide's window descriptor is read one
             // nuclide ahead (the record load depends on it)
@@ -472,7 +539,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, int roww, in
 // The S path for one warp's kLpl x 32 lookups (act: lane has a lookup; mat per lookup): an
 // optional warp energy sort, then one staged_material round per material among them.
 template <int GRID, bool OUTS>
-__device__ __forceinline__ void warp_lookups(const GridView &gv, const WarpStage &ws, bool (&act)[kLpl],
+__device__ __forceinline__ void warp_lookups(const GridView &gv, unsigned &tma_phase, const WarpStage &ws, bool (&act)[kLpl],
                                              double (&q)[kLpl], uint32_t (&r)[kLpl], int (&mat)[kLpl],
                                              int32_t *__restrict__ out_idx, Acc (&A)[kLpl])
 {
@@ -533,7 +600,7 @@ __device__ __forceinline__ void warp_lookups(const GridView &gv, const WarpStage
             mine[l] = act[l] && mat[l] == mat_w;
             todo[l] &= ~__ballot_sync(0xffffffffu, mine[l]);
         }
-        staged_material<GRID, OUTS>(gv, mat_w * gv.max_nucs, __ldg(gv.num_nucs + mat_w), mine, q, r, ws,
+        staged_material<GRID, OUTS>(gv, tma_phase, mat_w * gv.max_nucs, __ldg(gv.num_nucs + mat_w), mine, q, r, ws,
                                     out_idx, A);
     }
 }
@@ -552,6 +619,12 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
     __syncthreads();
     const WarpStage ws = warp_stage(st_smem);
     const int lane = threadIdx.x & 31;
+    unsigned tma_phase = 0; // XS_S_TMA: parity of the warp's mbarrier phase to wait for
+    if (kTma<GRID>) {
+        if (lane == 0)
+            mbar_init(ws.mbar);
+        __syncwarp();
+    }
     const uint64_t pol = policy_evict_first();
     uint32_t my_hash = 0, my_pairs = 0;
     for (;;) {
@@ -593,7 +666,7 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
                 q[l] = act[l] ? (so.q ? ld_stream(so.q + j, pol) : ld_stream(so.q_of + r[l], pol)) : 0.0;
                 mat[l] = !act[l] ? 0 : (one_mat ? mw : material_of(s_mb, (uint32_t)j));
             }
-            warp_lookups<GRID, OUTS>(gv, ws, act, q, r, mat, out_idx, A);
+            warp_lookups<GRID, OUTS>(gv, tma_phase, ws, act, q, r, mat, out_idx, A);
 #pragma unroll
             for (int l = 0; l < kLpl; l++) {
                 if (act[l]) {

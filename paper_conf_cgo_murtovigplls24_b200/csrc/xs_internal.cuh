@@ -38,6 +38,10 @@ constexpr int kMaxEnergyBins = 4096;
 #endif
 // XS_IV: lookups interpolate from per-interval records (iv) instead of point pairs (pts)
 constexpr bool kIv = XS_IV;
+#ifndef XS_S_TMA
+#define XS_S_TMA 1
+#endif
+constexpr bool kTmaStage = XS_S_TMA; // XS_SEARCH_S stages interval records with cp.async.bulk
 #ifndef XS_HASH_FAST
 #define XS_HASH_FAST 1
 #endif
@@ -81,6 +85,10 @@ struct Grid {
     // X_c[L+1]-X_c[L]) for c = 0..4} -- the differences the interpolation needs, rounded
     // once at build time exactly as the lookup would round them (XS_IV)
     double *iv = nullptr;
+    // ivs [n_nuc][n-1][14] (XS_S_TMA): the staged kernel's 112 B interval record
+    // {E_hi, 0, d = E_hi - E_lo, RN(1/d), (X_c,hi, X_c,hi - X_c,lo) x 5}, copied into shared
+    // memory by the bulk-copy engine (cp.async.bulk) instead of assembled by the warp
+    double *ivs = nullptr;
     // separator tree of every nuclide row (XS_SEARCH_W): level d has
     // 17^d nodes of 16 keys; node keys are E at base + (t+1)*stride[d] (+inf past n)
     double *tkeys = nullptr;
@@ -165,6 +173,7 @@ struct GridView {
     const double *__restrict__ E;
     const double *__restrict__ pts;
     const double *__restrict__ iv;
+    const double *__restrict__ ivs;
     const double *__restrict__ U;
     const int32_t *__restrict__ IDX;
     const int32_t *__restrict__ H;
