@@ -29,6 +29,9 @@ constexpr int kSortTpb = 1024;
 #ifndef XS_SCATTER_VEC
 #define XS_SCATTER_VEC 1
 #endif
+#ifndef XS_SCATTER_ILP4
+#define XS_SCATTER_ILP4 1
+#endif
 constexpr int64_t kScatterWindow = int64_t(64) << 20; // max bytes of slots one scatter launch writes
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
@@ -232,6 +235,19 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int
             slot_of[atomicAdd(&sh[k1], 1u)] = (uint32_t)(j0 + 1);
     };
     int v = threadIdx.x;
+#if XS_SCATTER_ILP4
+    // four 16 B key loads in flight per thread (the window's keys are a sparse 1/nwin of the
+    // stream: the kernel waits on these loads, ncu long_scoreboard 54%)
+    for (; v + 3 * kSortTpb < nvec; v += 4 * kSortTpb) {
+        const uint4 a = __ldg(kv + v), b = __ldg(kv + v + kSortTpb);
+        const uint4 c = __ldg(kv + v + 2 * kSortTpb), d = __ldg(kv + v + 3 * kSortTpb);
+        const int ja = beg + 8 * v, jb = ja + 8 * kSortTpb, jc = jb + 8 * kSortTpb, jd = jc + 8 * kSortTpb;
+        put(a.x, ja); put(a.y, ja + 2); put(a.z, ja + 4); put(a.w, ja + 6);
+        put(b.x, jb); put(b.y, jb + 2); put(b.z, jb + 4); put(b.w, jb + 6);
+        put(c.x, jc); put(c.y, jc + 2); put(c.z, jc + 4); put(c.w, jc + 6);
+        put(d.x, jd); put(d.y, jd + 2); put(d.z, jd + 4); put(d.w, jd + 6);
+    }
+#endif
     for (; v + kSortTpb < nvec; v += 2 * kSortTpb) {
         const uint4 a = __ldg(kv + v), b = __ldg(kv + v + kSortTpb);
         const int ja = beg + 8 * v, jb = ja + 8 * kSortTpb;
