@@ -322,7 +322,15 @@ constexpr int kRefineBins = XS_REFINE_BINS;         // B x S
 constexpr int kRefineTarget = kRefineCap * 5 / 8;   // mean slots per group the plan aims at
 static_assert(kRefineBins < 2048 && kRefineCap < (1 << 21), "bin and rank are packed into 11 + 21 bits");
 constexpr int kRefineMaxB = 64;
-constexpr int kJumpBytes = 4;                       // lookup offsets < 2^32
+// jump tables for lookup offsets j < 2^28 (kChunkSorted): digit t of j (widths 10, 9, 9 bits)
+// indexes table t, J(2 d 2^(shift t)); three table maps per energy instead of four byte maps
+// (and no padding slots, below: refine 1.09 -> 0.94 ms on large-U)
+constexpr int kJumpDigits = 3;
+__host__ __device__ constexpr int jump_bits(int t) { return t == 0 ? 10 : 9; }
+__host__ __device__ constexpr int jump_shift(int t) { return t == 0 ? 0 : (t == 1 ? 10 : 19); }
+__host__ __device__ constexpr int jump_base(int t) { return t == 0 ? 0 : (t == 1 ? 1024 : 1536); }
+constexpr int kJumpEntries = 2048;
+static_assert(jump_shift(2) + jump_bits(2) == 28, "the tables cover offsets < 2^28");
 
 // sub-bin of a lookup from its 63-bit stream state u (q = RN(u) 2^-63): the integer form of
 // floor((q nb - b) S), v = (u >> 20) nb ~ q nb 2^43 (< 2^59); rounding at the bucket edges
@@ -336,14 +344,14 @@ __device__ __forceinline__ int refine_bin(uint64_t u, uint32_t nb, int b, int kb
     return (kb << s_log2) + t;
 }
 
-// stream state of lookup offset j after its energy draw (sample_lookup: q = RN(u) 2^-63): the
-// byte maps applied to the chunk's base state one after the other (an offset byte of 0 maps
-// through the identity)
+// stream state of lookup offset j (< 2^28) after its energy draw (sample_lookup: q = RN(u)
+// 2^-63): the digit maps applied to the chunk's base state one after the other (a digit of 0
+// maps through the identity)
 __device__ __forceinline__ uint64_t energy_state(const Affine *jt, uint64_t s, uint32_t j)
 {
 #pragma unroll
-    for (int t = 0; t < kJumpBytes; t++) {
-        const Affine m = jt[t * 256 + ((j >> (8 * t)) & 255)];
+    for (int t = 0; t < kJumpDigits; t++) {
+        const Affine m = jt[jump_base(t) + ((j >> jump_shift(t)) & ((1u << jump_bits(t)) - 1))];
         s = m.a * s + m.c;
     }
     return lcg_step(s & kMod63);
@@ -358,8 +366,8 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
 {
     pdl_wait();
     pdl_trigger();
-    __shared__ Affine s_jt[kJumpBytes * 256];
-    __shared__ uint32_t s_hist[kRefineBins + 1]; // + a dummy bin for the slots past the group
+    __shared__ Affine s_jt[kJumpEntries];
+    __shared__ uint32_t s_hist[kRefineBins];
     __shared__ uint32_t s_bs[kRefineMaxB + 1]; // slot bounds of the group's buckets
     __shared__ uint32_t s_nbm[kRefineMaxB];
     __shared__ int s_b[kRefineMaxB];
@@ -369,7 +377,7 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
     uint32_t *s_r = reinterpret_cast<uint32_t *>(s_q + kRefineCap);
     const int K = bp.K;
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-    for (int i = tid; i < kJumpBytes * 256; i += kRefineTpb)
+    for (int i = tid; i < kJumpEntries; i += kRefineTpb)
         s_jt[i] = jt_g[i];
     const int ngroups = (K + B - 1) / B;
     for (int grp = blockIdx.x; grp < ngroups; grp += gridDim.x) {
@@ -403,8 +411,9 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
         double q[kRefinePer];
         int bin[kRefinePer];
         if (regs) {
-            // branch-free: positions past the group go to the dummy bin kRefineBins, whose
-            // slots (n, n + 1, ... < kRefineCap) are never written out
+            // positions past the group (the group holds ~2/3 of kRefineCap on average) skip the
+            // energy, bin and atomic: slot u of a warp's lanes is 32 consecutive positions, so
+            // the branch is warp-uniform except in one warp
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
                 const uint32_t t = s0 + tid + u * kRefineTpb;
@@ -413,14 +422,19 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
                 const uint32_t t = s0 + tid + u * kRefineTpb;
-                const uint64_t st = energy_state(s_jt, s_base, r[u]);
-                q[u] = u63_to_double(st);
-                const int bb = bin_of(t, st);
-                const int b = t < s1 ? bb : kRefineBins;
-                // the slot's rank inside its bin from the histogram atomic itself, packed above
-                // the bin index (bin < 2^11, rank < kRefineCap < 2^21): the placement below
-                // needs no second atomic (sort 0.406 -> 0.384 ms small, 2.47 -> 2.41 large-U)
-                bin[u] = b | (int)(atomicAdd(&s_hist[b], 1u) << 11);
+                if (t < s1) {
+                    const uint64_t st = energy_state(s_jt, s_base, r[u]);
+                    q[u] = u63_to_double(st);
+                    const int b = bin_of(t, st);
+                    // the slot's rank inside its bin from the histogram atomic itself, packed
+                    // above the bin index (bin < 2^11, rank < kRefineCap < 2^21): the placement
+                    // below needs no second atomic (sort 0.406 -> 0.384 ms small, 2.47 -> 2.41
+                    // large-U)
+                    bin[u] = b | (int)(atomicAdd(&s_hist[b], 1u) << 11);
+                } else {
+                    q[u] = 0.0;
+                    bin[u] = -1;
+                }
             }
         } else {
             for (uint32_t t = s0 + tid; t < s1; t += kRefineTpb)
@@ -460,14 +474,12 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
                 s_hist[k] = carry + incl - x;
             carry += __shfl_sync(0xffffffffu, incl, 31);
         }
-        if (tid == 0)
-            s_hist[kRefineBins] = s1 - s0;
         __syncthreads();
         if (regs) {
 #pragma unroll
             for (int u = 0; u < kRefinePer; u++) {
-                const uint32_t pos = s_hist[bin[u] & 2047] + ((uint32_t)bin[u] >> 11);
-                if (pos < (uint32_t)kRefineCap) {
+                if (bin[u] >= 0) {
+                    const uint32_t pos = s_hist[bin[u] & 2047] + ((uint32_t)bin[u] >> 11);
                     s_r[pos] = r[u];
                     s_q[pos] = q[u];
                 }
@@ -514,11 +526,11 @@ static void ensure_sort_space(Grid &g, int64_t chunk, int ctas, int K)
         XS_CUDA_TRY(cudaMalloc(&g.skey, (size_t)chunk * sizeof(uint16_t)));
         g.cap = chunk;
     }
-    if (!g.jt) { // byte jump tables of k_bucket_refine: jt[t][d] = J(2 d 256^t)
-        static Affine h[kJumpBytes * 256];
-        for (int t = 0; t < kJumpBytes; t++)
-            for (int d = 0; d < 256; d++)
-                h[t * 256 + d] = lcg_jump(2 * (uint64_t)d << (8 * t));
+    if (!g.jt) { // digit jump tables of k_bucket_refine: jt[base t + d] = J(2 d 2^(shift t))
+        static Affine h[kJumpEntries];
+        for (int t = 0; t < kJumpDigits; t++)
+            for (int d = 0; d < (1 << jump_bits(t)); d++)
+                h[jump_base(t) + d] = lcg_jump(2 * ((uint64_t)d << jump_shift(t)));
         XS_CUDA_TRY(cudaMalloc(&g.jt, sizeof(h)));
         XS_CUDA_TRY(cudaMemcpy(g.jt, h, sizeof(h), cudaMemcpyHostToDevice));
     }

@@ -118,7 +118,7 @@ struct Grid {
     uint32_t *si = nullptr;          // lookup offsets in (material, energy) order  [cap]
     uint16_t *skey = nullptr;        // bucket key by lookup offset                [cap]
     double *qs = nullptr;            // energies in (material, energy) order       [cap]
-    Affine *jt = nullptr;            // refine: byte jump tables J(2 d 256^t), [4][256]
+    Affine *jt = nullptr;            // refine: digit jump tables (sort.cu energy_state)
     uint32_t *si2 = nullptr;         // refine: the coarse slot order before k_bucket_refine [cap]
     int32_t *Lbuf = nullptr;         // split path: lower index of every pair      [lcap]
     int64_t lcap = 0;
