@@ -33,6 +33,11 @@ constexpr int kSortTpb = 1024;
 #define XS_SCATTER_ILP4 1
 #endif
 constexpr int64_t kScatterWindow = int64_t(64) << 20; // max bytes of slots one scatter launch writes
+#ifndef XS_SCATTER_ZERO
+#define XS_SCATTER_ZERO 1
+#endif
+constexpr bool kScatterZero = XS_SCATTER_ZERO;
+constexpr int64_t kZeroMinBytes = int64_t(96) << 20; // slot arrays above this get pre-zeroed windows
 
 __global__ void __launch_bounds__(kSortTpb) k_bucket_count(SampleView sv, BucketPlan bp, int per_cta, Affine J_tpb,
                                                             uint32_t *__restrict__ hist, double *__restrict__ q_of,
@@ -282,6 +287,32 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int
             slot_of[atomicAdd(&sh[k], 1u)] = (uint32_t)j;
     }
 #endif
+}
+
+// Zero the slots [base[klo], base[khi]) of the next scatter window with whole 16 B stores: the
+// L2 then holds the window's lines before the scatter's 4 B writes arrive, instead of reading
+// every sector from DRAM on its first partial write (the scatter's DRAM reads were ~the
+// window's size on top of the keys)
+__global__ void __launch_bounds__(1024) k_zero_window(int K, int klo, int khi, int count,
+                                                      const uint32_t *__restrict__ base, uint32_t *__restrict__ slot_of)
+{
+    pdl_wait();
+    pdl_trigger();
+    const uint32_t s0 = base[klo], s1 = khi < K ? base[khi] : (uint32_t)count;
+    const uint32_t a0 = (s0 + 3) & ~3u, a1 = s1 & ~3u; // 16 B aligned body
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (a0 < a1) {
+        uint4 *p = reinterpret_cast<uint4 *>(slot_of + a0);
+        const int64_t nv = (a1 - a0) >> 2;
+        for (int64_t i = t0; i < nv; i += stride)
+            p[i] = make_uint4(0, 0, 0, 0);
+    }
+    if (t0 < 8) { // the unaligned head and tail slots
+        const uint32_t j = t0 < 4 ? s0 + (uint32_t)t0 : a1 + (uint32_t)(t0 - 4);
+        if (t0 < 4 ? j < min(a0, s1) : (j >= max(a1, s0) && j < s1))
+            slot_of[j] = 0;
+    }
 }
 
 __global__ void k_bucket_gather(int count, const uint32_t *__restrict__ slot_of, const double *__restrict__ q_of,
@@ -610,8 +641,15 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, (cn * 4 + win_bytes - 1) / win_bytes));
     if (const char *env = std::getenv("XS_TEST_SCATTER_WINDOWS")) // test hook: force the window count
         nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, std::atoll(env)));
+    // pre-zero each window when the slot array exceeds the L2 (large-U / XL sort 2.16 / 2.76 ->
+    // 1.82 / 2.25 ms); an L2-sized one (17M lookups: 68 MB) is resident already and zeroing
+    // only adds work (small 0.337 -> 0.385 ms)
+    const bool zero = kScatterZero && (cn * 4 > kZeroMinBytes || std::getenv("XS_TEST_SCATTER_ZERO"));
     for (int w = 0; w < nwin; w++) {
         const int klo = (int)((int64_t)K * w / nwin), khi = (int)((int64_t)K * (w + 1) / nwin);
+        if (zero)
+            launch_pdl(k_zero_window, sms * 2, 1024, 0, stream, K, klo, khi, (int)cn, (const uint32_t *)g.base,
+                       refine ? g.si2 : g.si);
         launch_pdl(k_bucket_scatter, ctas, kSortTpb, (int)smem, stream, K, klo, khi, per_cta, (int)cn, g.hist, g.base,
                    g.skey, refine ? g.si2 : g.si);
     }
@@ -630,14 +668,14 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
                    lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), (const Affine *)g.jt,
                    (const uint32_t *)g.base, (const uint32_t *)g.si2, g.si, g.qs);
         XS_CUDA_TRY(cudaGetLastError());
-        return 4 + nwin;
+        return 4 + nwin * (zero ? 2 : 1);
     }
     if (post != kSortPostGather)
-        return 3 + nwin;
+        return 3 + nwin * (zero ? 2 : 1);
     const int gblocks = (int)std::min<int64_t>((cn + 255) / 256, (int64_t)sms * 8);
     k_bucket_gather<<<gblocks, 256, 0, stream>>>((int)cn, g.si, g.sq, g.qs);
     XS_CUDA_TRY(cudaGetLastError());
-    return 4 + nwin;
+    return 4 + nwin * (zero ? 2 : 1);
 }
 
 } // namespace xs

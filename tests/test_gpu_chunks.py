@@ -65,13 +65,18 @@ print("WINDOWS OK")
 """ % ROOT
 
 
+@pytest.mark.parametrize("zero", [False, True])
 @pytest.mark.parametrize("windows", [1, 2, 7, 39])
-def test_scatter_windows_match_oracle(windows):
+def test_scatter_windows_match_oracle(windows, zero):
     """the windowed scatter (one launch per window of buckets) with the window count forced
-    (XS_TEST_SCATTER_WINDOWS): every bucket is written by exactly one window"""
+    (XS_TEST_SCATTER_WINDOWS): every bucket is written by exactly one window; zero: each window
+    pre-zeroed first (k_zero_window, on by size for large sort chunks; XS_TEST_SCATTER_ZERO
+    forces it here, including windows whose slot range is not 16 B aligned)"""
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     env = dict(os.environ, XS_TEST_SCATTER_WINDOWS=str(windows))
+    if zero:
+        env["XS_TEST_SCATTER_ZERO"] = "1"
     r = subprocess.run([sys.executable, "-c", WINDOW_SCRIPT], capture_output=True, text=True, env=env, timeout=900)
     assert r.returncode == 0 and "WINDOWS OK" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
