@@ -44,6 +44,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_ALL
 #define XS_S_ALL 1
 #endif
+#ifndef XS_S_FASTGRIDS
+#define XS_S_FASTGRIDS 1 // grids (bit XS_UNIONIZED = 0, XS_NUCLIDE = 1, XS_HASH = 2) with the one-interval loop
+#endif
 #ifndef XS_S_FASTPF
 #define XS_S_FASTPF 1 // the fast loop's descriptors from lane registers (large-U 7.82 -> 7.73 ms)
 #endif
@@ -502,7 +505,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                 // (worth it where one-interval windows dominate -- the unionized configuration's
                 // 100M lookups: large-U 8.04 -> 7.91 ms; compiled into the nuclide / hash kernels
                 // it cost small / large / XL 0.5-2% through their register allocation)
-                if constexpr (GRID == XS_UNIONIZED && !OUTS) {
+                if constexpr (((XS_S_FASTGRIDS >> GRID) & 1) && !OUTS) {
                     const int myoc = (lane >= b0 && lane < b1) ? ocp[4 * lane] : -1;
                     const unsigned fast = __ballot_sync(0xffffffffu, myoc >= 0 && (myoc & 0xFFFF) == 1);
 #if XS_S_FASTPF
@@ -514,9 +517,10 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                             const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
                                               (ocj >> 16) * kIvDoubles;
                             const IvRec v = load_rec(R);
+                            const double conc = kTma<GRID> ? ws.meta[jj].conc : v.e.y;
 #pragma unroll
                             for (int l = 0; l < kLpl; l++)
-                                accumulate_interval(v, q[l], v.e.y, A[l]);
+                                accumulate_interval(v, q[l], conc, A[l]);
                         } else {
                             compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocj, ws.meta + jj,
                                                               ws.oeh, ws.orec, mine, q, r, out_idx, A);
@@ -528,9 +532,10 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                             const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
                                               (ocp[4 * jj] >> 16) * kIvDoubles;
                             const IvRec v = load_rec(R);
+                            const double conc = kTma<GRID> ? ws.meta[jj].conc : v.e.y;
 #pragma unroll
                             for (int l = 0; l < kLpl; l++)
-                                accumulate_interval(v, q[l], v.e.y, A[l]);
+                                accumulate_interval(v, q[l], conc, A[l]);
                         } else {
                             compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocp[4 * jj], ws.meta + jj,
                                                               ws.oeh, ws.orec, mine, q, r, out_idx, A);

@@ -1,5 +1,10 @@
 """compute-sanitizer over the tiny configuration: memcheck, racecheck,
-initcheck and synccheck on every kernel of grid creation, sorting and lookup."""
+initcheck and synccheck on every kernel of grid creation, sorting and lookup.
+
+Opt-in (XS_SANITIZER=1): the GPU pool this repo is tested on has closed compute-sanitizer (runs
+under it left GPUs needing a reset), and its wrapper refuses with exit code 86.  The round-1
+runs were clean with all four tools (profiles/r01*_gpu_tests.log); tests/test_gpu_guard.py
+checks with canary regions that no kernel writes outside the caller's buffers."""
 import os
 import subprocess
 import sys
@@ -30,6 +35,8 @@ print("SANITIZED")
 
 @pytest.mark.parametrize("tool", ["memcheck", "racecheck", "initcheck", "synccheck"])
 def test_compute_sanitizer(tool):
+    if os.environ.get("XS_SANITIZER") != "1":
+        pytest.skip("opt-in: XS_SANITIZER=1 (compute-sanitizer is closed on the GPU pool)")
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not installed")
     import torch
@@ -39,6 +46,8 @@ def test_compute_sanitizer(tool):
     if tool == "memcheck":
         args += ["--leak-check", "no"]
     r = subprocess.run(args + [sys.executable, "-c", SCRIPT], capture_output=True, text=True, timeout=1800)
+    if r.returncode == 86 and "closed" in r.stderr:
+        pytest.skip("compute-sanitizer refused on this pool: " + r.stderr.strip()[:200])
     assert r.returncode == 0 and "SANITIZED" in r.stdout, (r.stdout[-3000:], r.stderr[-3000:])
     text = r.stdout + r.stderr
     assert "ERROR SUMMARY: 0 errors" in text or "(0 errors, 0 warnings)" in text, text[-2000:]
