@@ -44,6 +44,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_ALL
 #define XS_S_ALL 1
 #endif
+#ifndef XS_S_FASTPAIR
+#define XS_S_FASTPAIR 1 // one-interval nuclides in pairs (large-U lookup 7.72 -> 7.47 ms; quads 7.53)
+#endif
 #ifndef XS_S_FASTGRIDS
 #define XS_S_FASTGRIDS 1 // grids (bit XS_UNIONIZED = 0, XS_NUCLIDE = 1, XS_HASH = 2) with the one-interval loop
 #endif
@@ -508,7 +511,56 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                 if constexpr (((XS_S_FASTGRIDS >> GRID) & 1) && !OUTS) {
                     const int myoc = (lane >= b0 && lane < b1) ? ocp[4 * lane] : -1;
                     const unsigned fast = __ballot_sync(0xffffffffu, myoc >= 0 && (myoc & 0xFFFF) == 1);
-#if XS_S_FASTPF
+#if XS_S_FASTPAIR
+                    // two consecutive one-interval nuclides per iteration (their records are
+                    // adjacent in the stage): one loop test and one shuffle per pair
+                    for (int jj = b0; jj < b1;) {
+                        const int ocj = __shfl_sync(0xffffffffu, myoc, jj);
+#if XS_S_FASTPAIR >= 4
+                        if (((fast >> jj) & 15u) == 15u && jj + 3 < b1) {
+                            const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
+                                              (ocj >> 16) * kIvDoubles;
+#pragma unroll
+                            for (int u = 0; u < 4; u++) {
+                                const IvRec v = load_rec(R + u * kIvDoubles);
+#pragma unroll
+                                for (int l = 0; l < kLpl; l++)
+                                    accumulate_interval(v, q[l], v.e.y, A[l]);
+                            }
+                            jj += 4;
+                        } else
+#endif
+                        if (((fast >> jj) & 3u) == 3u && jj + 1 < b1) {
+                            const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
+                                              (ocj >> 16) * kIvDoubles;
+                            {
+                                const IvRec v = load_rec(R);
+#pragma unroll
+                                for (int l = 0; l < kLpl; l++)
+                                    accumulate_interval(v, q[l], v.e.y, A[l]);
+                            }
+                            {
+                                const IvRec v = load_rec(R + kIvDoubles);
+#pragma unroll
+                                for (int l = 0; l < kLpl; l++)
+                                    accumulate_interval(v, q[l], v.e.y, A[l]);
+                            }
+                            jj += 2;
+                        } else if ((fast >> jj) & 1u) {
+                            const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
+                                              (ocj >> 16) * kIvDoubles;
+                            const IvRec v = load_rec(R);
+#pragma unroll
+                            for (int l = 0; l < kLpl; l++)
+                                accumulate_interval(v, q[l], v.e.y, A[l]);
+                            jj++;
+                        } else {
+                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocj, ws.meta + jj,
+                                                              ws.oeh, ws.orec, mine, q, r, out_idx, A);
+                            jj++;
+                        }
+                    }
+#elif XS_S_FASTPF
                     // the descriptors of the pass are already in lane registers (myoc): the
                     // record address comes from a shuffle, not a dependent shared-memory load
                     for (int jj = b0; jj < b1; jj++) {
