@@ -67,8 +67,11 @@ def parse(argv=None):
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--workload", default="large-U", choices=sorted(WORKLOADS))
-    p.add_argument("--scaling", default="", choices=["", "strong", "weak"],
-                   help="default: the workload's (XL weak at 125M per rank, the rest strong)")
+    p.add_argument("--scaling", default="", choices=["", "strong", "weak", "strong-index"],
+                   help="default: the workload's (XL weak at 125M per rank, the rest strong). strong: "
+                        "key-range shards (every rank draws the whole range and looks up its share of the "
+                        "(material, energy) buckets, DESIGN.md §9); strong-index: index ranges "
+                        "[floor(rT/N), floor((r+1)T/N)) (SURVEY.md §8e)")
     p.add_argument("--lookups", type=int, default=0, help="override: job total (strong) or per rank (weak)")
     p.add_argument("--search", default="S")
     p.add_argument("--sort", default="material_energy")
@@ -86,19 +89,26 @@ def parse(argv=None):
 
 # ------------------------------------------------------------------ sizes and rooflines
 def scaling_of(a, w) -> str:
+    """strong (key-range shards), strong-index or weak"""
     return a.scaling or w.scaling
 
 
+def scaling_kind(scaling: str) -> str:
+    """the contract's `scaling` field: strong or weak"""
+    return "weak" if scaling == "weak" else "strong"
+
+
 def rank_range(w, scaling: str, total_override: int, rank: int, world: int):
-    """(first, count) of this rank."""
+    """(first, count) of this rank's index range: strong splits the job's total,
+    weak gives every rank its own per-rank count"""
     from paper_conf_cgo_murtovigplls24_b200 import driver
     n = total_override or w.lookups
-    return driver.shard(n, rank, world) if scaling == "strong" else driver.weak_range(n, rank)
+    return driver.shard(n, rank, world) if scaling_kind(scaling) == "strong" else driver.weak_range(n, rank)
 
 
 def job_lookups(w, scaling: str, total_override: int, world: int) -> int:
     n = total_override or w.lookups
-    return n if scaling == "strong" else n * world
+    return n if scaling_kind(scaling) == "strong" else n * world
 
 
 def algorithmic_bytes_per_lookup(w) -> float:
@@ -297,9 +307,11 @@ class Clocks:
 def config_of(a, w, world: int) -> dict:
     """The workload `config` both arms print (identical, so the driver can pair them)."""
     sc = scaling_of(a, w)
+    split = ("key-range shards: every rank draws all lookups, orders and looks up its 1/N of the "
+             "(material, energy) buckets by expected cost" if sc == "strong" and world > 1 else "lookup index ranges")
     return {"workload": w.name, "n_nuclides": w.n_nuclides, "n_gridpoints": w.n_gridpoints,
             "grid": GRID_NAMES[w.grid_type], "lookups_total": job_lookups(w, sc, a.lookups, world),
-            "scaling": sc, "l2_flush": not a.no_flush, "parallelism": f"dp{world} (lookup index ranges)"}
+            "scaling": scaling_kind(sc), "l2_flush": not a.no_flush, "parallelism": f"dp{world} ({split})"}
 
 
 def cpu_baseline(w, lookups_cap: int, seconds: float):
@@ -356,7 +368,7 @@ def run_reference(a, w):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * tsum / len(times),
-        "higher_is_better": True, "scaling": scaling_of(a, w), "vs_baseline": None, "dtype": "f64",
+        "higher_is_better": True, "scaling": scaling_kind(scaling_of(a, w)), "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (XSBench LCG grid + lookups, seeds 42/1070)",
         "config": config_of(a, w, world),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
@@ -377,15 +389,26 @@ class Runner:
         from paper_conf_cgo_murtovigplls24_b200 import driver
         self.torch, self.xs, self.driver, self.a, self.w, self.R = torch, xs, driver, a, w, R
         self.scaling = scaling
+        # index range of this rank (weak, strong-index, and the passes key shards do not serve)
         self.first, self.count = rank_range(w, scaling, a.lookups, R.rank, R.world)
         self.total = int(driver.sum_over_ranks(self.count))
+        # strong at N > 1: key-range shard (rank, N) of the whole range [0, total)
+        self.keys = scaling == "strong" and R.world > 1
         self.g = xs.Grid(w.n_nuclides, w.n_gridpoints, w.grid_type, GRID_SEED)
         assert driver.replicas_identical(self.g.checksum()), "grid replicas differ across ranks"
         self.stream = torch.cuda.current_stream()
         self.flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=self.g.device)
         self.opts = dict(search=a.search, sort=a.sort, energy_bins=a.energy_bins, timing=True)
 
+    def uses_keys(self, o) -> bool:
+        """key-range shards serve the refined order with the staged kernel (xs.h)"""
+        oo = {**self.opts, **o}
+        return self.keys and oo["search"] == "S" and oo["sort"] == "material_energy" and not oo.get("coarse")
+
     def step(self, **o):
+        if self.uses_keys(o):
+            return self.g.lookup_range(0, self.total, LOOKUP_SEED, None,
+                                       **{**self.opts, **o, "shard": (self.R.rank, self.R.world)})
         return self.g.lookup_range(self.first, self.count, LOOKUP_SEED, None, **{**self.opts, **o})
 
     def timed(self, k_steps, warm, **o):
@@ -407,9 +430,14 @@ class Runner:
         ms = [s_.elapsed_time(e_) for s_, e_ in evs]
         return ms, out, self.driver.max_over_ranks(sum(ms))
 
-    def golden(self, stats):
-        """Every rank's hash and pairs against the oracle's golden eighths; True/False/None
-        (None: the split does not fall on the golden boundaries)."""
+    def golden(self, stats, keys=False):
+        """Index ranges: every rank's hash and pairs against the oracle's golden eighths; key
+        shards: the sums over ranks against the golden total of the whole range.  True / False
+        / None (None: the split does not fall on the golden boundaries)."""
+        if keys:
+            h, nl, pr, _ = self.driver.reduce_stats(stats.hash, stats.lookups, stats.pairs, 0.0)
+            exp = golden_expect(self.w.name, 0, self.total)
+            return None if exp is None else bool(h == exp[0] and pr == exp[1] and nl == self.total)
         exp = golden_expect(self.w.name, self.first, self.count)
         ok = -1 if exp is None else int(stats.hash == exp[0] and stats.pairs == exp[1])
         lo = self.driver.min_over_ranks(ok)
@@ -425,12 +453,14 @@ def summarize(run: Runner, ms_max, stats, steps, sms, clocks=None, **o):
     lookup_ms = statistics.mean(x.lookup_ms for x in stats)
     search = o.get("search", run.a.search)
     sort = o.get("sort", run.a.sort)
+    keys = run.uses_keys(o)
     return {"value": run.total * steps / (ms_max / 1e3), "ms_per_step": ms_max / steps,
-            "lookups_per_gpu": run.count, "sort_ms": statistics.mean(x.sample_ms for x in stats),
+            "lookups_per_gpu": int(s0.lookups), "sort_ms": statistics.mean(x.sample_ms for x in stats),
             "lookup_ms": lookup_ms, "hash": h, "pairs": npairs, "lookups": nl,
+            "split": "key-range shards" if keys else "index ranges",
             "hash_consistent": all(x.hash == s0.hash for x in stats),
-            "golden_match": run.golden(s0),
-            "roofline": roofline(run.w, search, sort, run.count, s0.pairs, lookup_ms, sms, clocks)}
+            "golden_match": run.golden(s0, keys),
+            "roofline": roofline(run.w, search, sort, int(s0.lookups), s0.pairs, lookup_ms, sms, clocks)}
 
 
 def run_ours(a, w):
@@ -457,7 +487,8 @@ def run_ours(a, w):
                      ("U2 XSBench order (unsorted)", dict(search="U2", sort="none"))):
         ms, sts, mx = run.timed(a.ab_steps, 2, **o)
         north[label] = summarize(run, mx, sts, a.ab_steps, sms, **o)
-        north[label]["hash_ok"] = all(x.hash == stats[0].hash for x in sts)
+        # the job's hash (reduced over ranks) is the same whatever the split or search
+        north[label]["hash_ok"] = north[label]["hash"] == main["hash"] and north[label]["hash_consistent"]
 
     # ---- the paper's A/B on this workload: every search variant, same protocol, fewer steps
     ab = {}
@@ -467,9 +498,10 @@ def run_ours(a, w):
              ("M/unsorted (XSBench order)", dict(search="M", sort="none"))] if variants else []
     for label, o in [(v, dict(search=v)) for v in variants] + extra:
         ms, sts, mx = run.timed(a.ab_steps, 2, **o)
+        h_job = driver.reduce_stats(sts[0].hash, sts[0].lookups, sts[0].pairs, 0.0)[0]
         ab[label] = {"value": run.total * a.ab_steps / (mx / 1e3), "sort_ms": statistics.mean(x.sample_ms for x in sts),
                      "lookup_ms": statistics.mean(x.lookup_ms for x in sts),
-                     "hash_ok": all(x.hash == stats[0].hash for x in sts)}
+                     "hash_ok": h_job == main["hash"] and all(x.hash == sts[0].hash for x in sts)}
 
     # ---- e2e: the public API with HOST output buffers (D2H of every macro XS in the region)
     e2e = None
@@ -497,13 +529,14 @@ def run_ours(a, w):
             if R.world == 1:
                 run.xs.xs_lookup_batch(run.g.handle, run.count, LOOKUP_SEED, None)
             else:
-                run.g.lookup_range(run.first, run.count, LOOKUP_SEED, None, search=a.search, sort=a.sort)
+                run.step(timing=False)
             th.append(time.perf_counter() - t0)
         e2e_h = driver.max_over_ranks(sum(th))
         e2e = {"value": run.total * len(t) / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 0,
                "d2h_bytes_per_step": run.count * 5 * 8 + 16,
                "note": "xs_lookup_range writing every macroscopic XS into pinned HOST memory (D2H "
-                       "overlapped with compute in 4M-lookup chunks), host wall clock, max over ranks; "
+                       "overlapped with compute in 4M-lookup chunks; each rank its index range -- key-range "
+                       "shards write device memory only), host wall clock, max over ranks; "
                        "inputs are the (seed, range) scalars -- lookups are drawn on device by the "
                        "method's counter-based LCG (DESIGN.md §8)",
                "hash_only": {"value": run.total * len(th) / e2e_h, "d2h_bytes_per_step": 16,
@@ -536,7 +569,7 @@ def run_ours(a, w):
     line = {
         "metric": METRIC, "value": main["value"], "unit": UNIT, "n_gpus": R.world, "steps": a.steps,
         "warmup": a.warmup, "ms_per_step": main["ms_per_step"], "higher_is_better": True,
-        "scaling": scaling, "vs_baseline": None, "dtype": "f64",
+        "scaling": scaling_kind(scaling), "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (XSBench LCG grid + lookups, seeds 42/1070)",
         "config": config_of(a, w, R.world),
         "path": {"search": a.search, "sort": a.sort, "backend": driver.backend_name(),
@@ -547,7 +580,8 @@ def run_ours(a, w):
         "roofline": main["roofline"],
         "verification": {"hash": main["hash"], "lookups": main["lookups"], "pairs": main["pairs"],
                          "golden_match": main["golden_match"], "hash_consistent": main["hash_consistent"],
-                         "golden": "tests/golden/hashes.json (CPU oracle, every rank's range)"},
+                         "golden": "tests/golden/hashes.json (CPU oracle: every rank's index range, or the "
+                                   "ranks' sum over the whole range for key-range shards)"},
         "north_star": north,
         "workloads": workloads,
         "ab": ab,

@@ -116,6 +116,19 @@ typedef struct xs_opts {
                             material's expected (lookup, nuclide) pairs                 */
     uint32_t flags;      /* XS_FLAG_*                                                   */
     int32_t history_len; /* XS_SORT_HISTORY: lookups per particle; 0 = default (34)     */
+    int32_t shard_index; /* key-range sharding (XS_SORT_MATERIAL_ENERGY + XS_SEARCH_S, the
+                            refined order; a strong-scaling split of one lookup range over
+                            shard_count processes): the call draws EVERY lookup
+                            of [first, first + count) but orders and looks up only those whose
+                            (material, energy) bucket lies in the shard_index-th of
+                            shard_count equal bucket ranges -- each shard then holds ~count /
+                            shard_count lookups at the full range's energy density.  stats
+                            cover the shard's lookups (stats.lookups = how many); rows of
+                            out_macro_xs (device memory only; out_idx unsupported) of the
+                            other lookups are left untouched.
+                            The shards' hashes, pairs and lookups sum to the unsharded call's.
+                            0 <= shard_index < shard_count                              */
+    int32_t shard_count; /* 0 or 1 = no sharding (the default)                          */
 } xs_opts;
 
 typedef struct xs_stats {

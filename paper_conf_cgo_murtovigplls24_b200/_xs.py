@@ -45,7 +45,7 @@ BZ_NAMES = {"M": 0, "M2": 1, "U1": 2, "U2": 3, "S": 4, "T": 5}
 class xs_opts(C.Structure):
     _fields_ = [("search", C.c_int32), ("sort", C.c_int32), ("stream", C.c_void_p),
                 ("block", C.c_int32), ("energy_bins", C.c_int32), ("flags", C.c_uint32),
-                ("history_len", C.c_int32)]
+                ("history_len", C.c_int32), ("shard_index", C.c_int32), ("shard_count", C.c_int32)]
 
 
 class xs_stats(C.Structure):

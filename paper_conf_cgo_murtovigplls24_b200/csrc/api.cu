@@ -73,6 +73,8 @@ void xs_opts_default(xs_opts *o)
     o->energy_bins = 0;
     o->flags = 0;
     o->history_len = 0;
+    o->shard_index = 0;
+    o->shard_count = 1;
 }
 
 const char *xs_last_error(void) { return t_err.c_str(); }

@@ -686,10 +686,11 @@ __device__ __forceinline__ void warp_lookups(const GridView &gv, unsigned &tma_p
 
 template <int GRID, bool OUTS>
 __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
-    k_lookup_staged(GridView gv, SortedView so, int count, double *__restrict__ out_, int32_t *__restrict__ out_idx_,
+    k_lookup_staged(GridView gv, SortedView so, int count_arg, double *__restrict__ out_, int32_t *__restrict__ out_idx_,
                     unsigned long long *__restrict__ stats)
 {
     pdl_wait(); // the sort's outputs (and the work counter it zeroed) are complete
+    const int count = so.count_dev ? (int)*so.count_dev : count_arg; // a key-range shard's slots
     double *__restrict__ out = OUTS ? out_ : nullptr;
     int32_t *__restrict__ out_idx = OUTS ? out_idx_ : nullptr;
     __shared__ uint32_t s_mb[kMaterials + 1];
@@ -762,10 +763,12 @@ __global__ void __launch_bounds__(kStTpb, XS_S_MIN_BLOCKS)
         __threadfence();
         if (atomicAdd(so.done, 1u) == gridDim.x - 1) {
             __threadfence();
-            const unsigned long long h = atomicAdd(stats + 0, 0ull), pr = atomicAdd(stats + 1, 0ull);
+            const unsigned long long h = atomicAdd(stats + 0, 0ull), pr = atomicAdd(stats + 1, 0ull),
+                                     nl = atomicAdd(stats + 2, 0ull);
             volatile unsigned long long *p = so.pub;
             p[0] = h;
             p[1] = pr;
+            p[2] = nl;
             __threadfence_system();
         }
     }

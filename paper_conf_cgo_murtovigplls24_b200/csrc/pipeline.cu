@@ -150,6 +150,16 @@ static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t see
     const bool history = o.sort == XS_SORT_HISTORY;
     const int hl = o.history_len ? o.history_len : 34;
     XS_CHECK_ARG(!history || (hl >= 1 && hl <= (1 << 20)), "opts.history_len must be in [1, 2^20]");
+    // key-range sharding (xs.h): the refined (material, energy) order with the staged kernel
+    const int nshards = o.shard_count > 1 ? o.shard_count : 1;
+    const int shard = nshards > 1 ? o.shard_index : 0;
+    const bool sharded = nshards > 1;
+    XS_CHECK_ARG(o.shard_count >= 0 && o.shard_index >= 0 && (o.shard_count <= 1 ? o.shard_index == 0 : shard < nshards),
+                 "opts.shard_index must be in [0, shard_count)");
+    XS_CHECK_ARG(!sharded || (o.sort == XS_SORT_MATERIAL_ENERGY && o.search == XS_SEARCH_S && o.energy_bins != 1 &&
+                              !(o.flags & (XS_FLAG_SPLIT | XS_FLAG_COARSE))),
+                 "key-range sharding needs sort = XS_SORT_MATERIAL_ENERGY, search = XS_SEARCH_S, no split / coarse");
+    XS_CHECK_ARG(!sharded || out_idx == nullptr, "key-range sharding does not write out_idx");
     const int tpb = o.block ? o.block : 256;
     XS_CHECK_ARG(tpb == 64 || tpb == 128 || tpb == 256, "opts.block must be 64, 128 or 256");
     const int nb = (o.sort == XS_SORT_MATERIAL_ENERGY) ? (o.energy_bins ? o.energy_bins : kMaxEnergyBins) : 1;
@@ -160,6 +170,7 @@ static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t see
     const bool sorted = o.sort == XS_SORT_MATERIAL || o.sort == XS_SORT_MATERIAL_ENERGY;
     const bool fused = !sorted || !(o.flags & XS_FLAG_SPLIT);
     const bool host_out = out_macro && !is_device_accessible(out_macro);
+    XS_CHECK_ARG(!sharded || !host_out, "key-range sharding writes device outputs only");
     int64_t chunk = fused ? (sorted ? kChunkSorted : kChunkFused) : kChunkSplit;
     if (host_out)
         chunk = std::min(chunk, kChunkHost);
@@ -197,7 +208,7 @@ static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t see
         XS_CUDA_TRY(cudaMallocHost(&g.mb_h, 32 * sizeof(uint32_t)));
 
     XS_CUDA_TRY(cudaEventRecord(g.ev[0], stream));
-    XS_CUDA_TRY(cudaMemsetAsync(g.stats_d, 0, 2 * sizeof(uint64_t), stream));
+    XS_CUDA_TRY(cudaMemsetAsync(g.stats_d, 0, 3 * sizeof(uint64_t), stream)); // hash, pairs, shard lookups
     if (out_idx && count > 0)
         XS_CUDA_TRY(cudaMemsetAsync(out_idx, 0xFF, (size_t)count * g.max_nucs * sizeof(int32_t), stream));
     unsigned long long *stats = (unsigned long long *)g.stats_d;
@@ -217,12 +228,13 @@ static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t see
             int K = 0;
             const bool refine = fused && o.sort == XS_SORT_MATERIAL_ENERGY && nb > 1 && !(o.flags & XS_FLAG_COARSE);
             launches += launch_bucket_sort(g, sv, nb, !fused ? kSortPostGather : (refine ? kSortPostRefine : kSortPostNone),
-                                           stream, &K);
+                                           stream, &K, shard, nshards, (unsigned long long *)(g.stats_d + 2));
             so.q = (!fused || refine) ? g.qs : nullptr; // q in slot order when the sort wrote it
             so.q_of = refine ? nullptr : g.sq;
             so.slot = g.si;
             so.mb_dev = g.base + K;
             so.work = reinterpret_cast<int *>(g.stats_d + 4); // zeroed by k_bucket_count
+            so.count_dev = sharded ? g.base + K + kMaterials : nullptr; // the shard's slots
             if (fused && o.search == XS_SEARCH_S && c0 + chunk >= count) { // the last chunk of S
                 so.done = reinterpret_cast<unsigned int *>(g.stats_d + 5);   // publishes the stats
                 so.pub = reinterpret_cast<unsigned long long *>(g.stats_h);
@@ -302,7 +314,7 @@ static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t see
         if (copied_pending[b])
             XS_CUDA_TRY(cudaStreamWaitEvent(stream, g.ev_copied[b], 0));
     if (!published || count == 0)
-        XS_CUDA_TRY(cudaMemcpyAsync(g.stats_h, g.stats_d, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, stream));
+        XS_CUDA_TRY(cudaMemcpyAsync(g.stats_h, g.stats_d, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, stream));
     XS_CUDA_TRY(cudaEventRecord(g.ev[6], stream));
     XS_CUDA_TRY(cudaStreamSynchronize(stream));
     float total = 0;
@@ -319,7 +331,7 @@ static void run_lookups_impl(Grid &g, int64_t first, int64_t count, uint64_t see
     if (st) {
         st->hash = g.stats_h[0];
         st->pairs = g.stats_h[1];
-        st->lookups = (uint64_t)count;
+        st->lookups = sharded ? g.stats_h[2] : (uint64_t)count;
         st->device_ms = total;
         st->sample_ms = sample_ms;
         st->lookup_ms = lookup_ms;

@@ -149,9 +149,13 @@ __global__ void __launch_bounds__(32 * kColWarps) k_bucket_colscan(int K, int ct
 
 // one CTA: exclusive scan of base[0..K) in place.  Warp w owns a contiguous segment and
 // walks it 32 coalesced elements at a time (warp scan + carry) -- no bank conflicts;
-// a block scan of the warp totals gives each warp its offset for the second pass.  Then
-// base[K + m] = first slot of material m, base[K + 12] = count.
-__global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, uint32_t *__restrict__ base)
+// a block scan of the warp totals gives each warp its offset for the second pass.  Then, for
+// the shard's buckets [kA, kB) (everything unsharded) whose slots are re-based to start at 0:
+// base[K + m] = first slot of material m in the shard (clamped to [0, n]), base[K + 12] = n,
+// the shard's lookups (also added to *n_acc), base[K + 13] = every bucket's total,
+// base[K + 14] = base[kA] (the slot the shard's slots are re-based by).
+__global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, int kA, int kB, uint32_t *__restrict__ base,
+                                                      unsigned long long *__restrict__ n_acc)
 {
     pdl_wait();
     pdl_trigger();
@@ -197,10 +201,23 @@ __global__ void __launch_bounds__(1024) k_bucket_base(BucketPlan bp, uint32_t *_
     }
     __syncthreads();
     if (threadIdx.x == 0) {
+        const uint32_t total = wsum[31];
+        const uint32_t s0 = kA < K ? base[kA] : total, s1 = kB < K ? base[kB] : total;
+        const uint32_t n = s1 - s0;
+        uint32_t mb[kMaterials];
+#pragma unroll
+        for (int m = 0; m < kMaterials; m++) {
+            const uint32_t b = bp.kbase[m] < K ? base[bp.kbase[m]] : total;
+            mb[m] = b <= s0 ? 0u : (b >= s1 ? n : b - s0);
+        }
 #pragma unroll
         for (int m = 0; m < kMaterials; m++)
-            base[K + m] = base[bp.kbase[m]];
-        base[K + kMaterials] = wsum[31];
+            base[K + m] = mb[m];
+        base[K + kMaterials] = n;
+        base[K + kMaterials + 1] = total;
+        base[K + kMaterials + 2] = s0;
+        if (n_acc)
+            atomicAdd(n_acc, (unsigned long long)n);
     }
 }
 
@@ -217,8 +234,9 @@ __global__ void __launch_bounds__(kSortTpb) k_bucket_scatter(int K, int klo, int
     pdl_trigger();
     extern __shared__ uint32_t sh[];
     const uint32_t *h = hist + (int64_t)blockIdx.x * K;
+    const uint32_t rebase = base[K + kMaterials + 2]; // the shard's first slot (0 unsharded)
     for (int k = klo + threadIdx.x; k < khi; k += kSortTpb)
-        sh[k] = base[k] + h[k];
+        sh[k] = base[k] + h[k] - rebase;
     __syncthreads();
     const int beg = blockIdx.x * per_cta;
     const int end = min(beg + per_cta, count);
@@ -298,7 +316,9 @@ __global__ void __launch_bounds__(1024) k_zero_window(int K, int klo, int khi, i
 {
     pdl_wait();
     pdl_trigger();
-    const uint32_t s0 = base[klo], s1 = khi < K ? base[khi] : (uint32_t)count;
+    const uint32_t rebase = base[K + kMaterials + 2], total = base[K + kMaterials + 1];
+    const uint32_t s0 = base[klo] - rebase, s1 = (khi < K ? base[khi] : total) - rebase;
+    (void)count;
     const uint32_t a0 = (s0 + 3) & ~3u, a1 = s1 & ~3u; // 16 B aligned body
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -388,7 +408,8 @@ __device__ __forceinline__ uint64_t energy_state(const Affine *jt, uint64_t s, u
     return lcg_step(s & kMod63);
 }
 
-__global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(BucketPlan bp, int B, int s_log2, int count,
+__global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(BucketPlan bp, int kA, int kB, int B,
+                                                                  int s_log2,
                                                                   uint64_t s_base, const Affine *__restrict__ jt_g,
                                                                   const uint32_t *__restrict__ base,
                                                                   const uint32_t *__restrict__ slot_in,
@@ -410,11 +431,13 @@ __global__ void __launch_bounds__(kRefineTpb, XS_REFINE_MINB) k_bucket_refine(Bu
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     for (int i = tid; i < kJumpEntries; i += kRefineTpb)
         s_jt[i] = jt_g[i];
-    const int ngroups = (K + B - 1) / B;
+    const int ngroups = (kB - kA + B - 1) / B;
+    // the shard's slots start at 0 (base[K + 14] = base[kA]; 0 and kA = 0 unsharded)
+    const uint32_t rebase = __ldg(base + K + kMaterials + 2), total = __ldg(base + K + kMaterials + 1);
     for (int grp = blockIdx.x; grp < ngroups; grp += gridDim.x) {
-        const int k0 = grp * B, nbk = min(B, K - k0);
+        const int k0 = kA + grp * B, nbk = min(B, kB - k0);
         if (tid <= nbk)
-            s_bs[tid] = (k0 + tid < K) ? __ldg(base + k0 + tid) : (uint32_t)count;
+            s_bs[tid] = ((k0 + tid < K) ? __ldg(base + k0 + tid) : total) - rebase;
         if (tid < nbk) {
             const int k = k0 + tid;
             int m = 0;
@@ -599,7 +622,45 @@ static BucketPlan make_plan(const Grid &g, int total, bool by_lookups)
     return bp;
 }
 
-int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out)
+// Key-range shard boundaries: shard s of n owns buckets [b(s), b(s+1)), b(s) the first bucket at
+// which the expected cost of the buckets before it reaches s/n of the total -- a bucket's
+// expected cost is its expected lookups (P(m) / nb[m] of the range) times (num_nucs[m] +
+// kShardLookupCost), so the fuel's buckets (81% of large's pairs in 14% of its lookups) are
+// spread over most shards.  Monotone in s, b(0) = 0, b(n) = K: the shards partition the buckets.
+#ifndef XS_SHARD_LOOKUP_COST
+#define XS_SHARD_LOOKUP_COST 22
+#endif
+constexpr double kShardLookupCost = XS_SHARD_LOOKUP_COST;
+
+static int shard_boundary(const Grid &g, const BucketPlan &bp, int s, int n)
+{
+    if (s <= 0)
+        return 0;
+    if (s >= n)
+        return bp.K;
+    double w[kMaterials], W = 0;
+    for (int m = 0; m < kMaterials; m++) {
+        const double p = (m == 0) ? 1.0 - g.thresholds[11] : g.thresholds[m] - g.thresholds[m - 1];
+        // expected cost of the material, spread evenly over its buckets: its pairs plus a
+        // per-lookup share (the sort's scatter and refine, the lookup kernel's per-warp window
+        // and staging work) worth ~kShardLookupCost pairs
+        w[m] = p * (g.num_nucs[m] + kShardLookupCost);
+        W += w[m];
+    }
+    const double target = W * s / n;
+    double cum = 0;
+    for (int m = 0; m < kMaterials; m++) {
+        if (cum + w[m] >= target && w[m] > 0) {
+            const int k = bp.kbase[m] + (int)std::ceil((target - cum) / (w[m] / bp.nb[m]) - 1e-9);
+            return std::min(std::max(k, bp.kbase[m]), bp.kbase[m + 1]);
+        }
+        cum += w[m];
+    }
+    return bp.K;
+}
+
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out,
+                       int shard, int nshards, unsigned long long *n_acc)
 {
     {
         const int bytes = kMaterials * kMaxEnergyBins * 4; // the largest histogram a plan can ask for
@@ -629,24 +690,31 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     launch_pdl(k_bucket_count, ctas, kSortTpb, (int)smem, stream, sv, bp, per_cta, J, g.hist,
                refine ? nullptr : g.sq, g.skey, (unsigned long long *)(g.stats_d + 4));
     launch_pdl(k_bucket_colscan, (K + 31) / 32, 32 * kColWarps, 0, stream, K, ctas, g.hist, g.base);
-    launch_pdl(k_bucket_base, 1, 1024, 0, stream, bp, g.base);
+    // key-range shard (xs_opts.shard_*): buckets [kA, kB) -- every lookup is drawn and counted,
+    // only the shard's are ordered (slots re-based to start at 0 by k_bucket_base)
+    const int kA = shard_boundary(g, bp, shard, nshards), kB = shard_boundary(g, bp, shard + 1, nshards);
+    const int64_t cn_own = (cn * (kB - kA) + K - 1) / K; // expected slots of the shard
+    launch_pdl(k_bucket_base, 1, 1024, 0, stream, bp, kA, kB, g.base, n_acc);
     // windows of ~equal expected slot counts (refine: equal-size buckets; coarse: cost-weighted
     // buckets, so the windows are only approximately equal)
-    // window: 1/6 of the slot array, within [16, 64] MB -- more windows keep each one's
-    // random writes more L2-local, but every window re-reads all 2 B keys (measured: 17M
-    // lookups best at 16 MB, 100M-125M at 48 MB; with the 16 B key loads at 64 MB, r01be)
-    int64_t win_bytes = std::min<int64_t>(kScatterWindow, std::max<int64_t>(int64_t(16) << 20, cn * 4 / 6));
+    // window: 1/6 of the slot array, at least 16 MB, and 64 MB once the slots exceed 128 MB --
+    // more windows keep each one's random writes more L2-local, but every window re-reads all
+    // 2 B keys (measured, sort ms with pre-zeroing: 25M lookups 16 MB 0.558 / 64 MB 0.613,
+    // 50M 33 MB 1.285 / 64 MB 1.126, 100M 64 MB 1.82, 125M 64 MB 2.25; profiles/r02n_mid2.jsonl)
+    int64_t win_bytes = cn_own * 4 > (int64_t(128) << 20)
+                            ? kScatterWindow
+                            : std::min<int64_t>(kScatterWindow, std::max<int64_t>(int64_t(16) << 20, cn_own * 4 / 6));
     if (const char *env = std::getenv("XS_SCATTER_WINDOW_MB"))
         win_bytes = std::max(1ll, std::atoll(env)) << 20;
-    int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, (cn * 4 + win_bytes - 1) / win_bytes));
+    int nwin = (int)std::max<int64_t>(1, std::min<int64_t>(kB - kA, (cn_own * 4 + win_bytes - 1) / win_bytes));
     if (const char *env = std::getenv("XS_TEST_SCATTER_WINDOWS")) // test hook: force the window count
-        nwin = (int)std::max<int64_t>(1, std::min<int64_t>(K, std::atoll(env)));
+        nwin = (int)std::max<int64_t>(1, std::min<int64_t>(kB - kA, std::atoll(env)));
     // pre-zero each window when the slot array exceeds the L2 (large-U / XL sort 2.16 / 2.76 ->
     // 1.82 / 2.25 ms); an L2-sized one (17M lookups: 68 MB) is resident already and zeroing
     // only adds work (small 0.337 -> 0.385 ms)
-    const bool zero = kScatterZero && (cn * 4 > kZeroMinBytes || std::getenv("XS_TEST_SCATTER_ZERO"));
+    const bool zero = kScatterZero && (cn_own * 4 > kZeroMinBytes || std::getenv("XS_TEST_SCATTER_ZERO"));
     for (int w = 0; w < nwin; w++) {
-        const int klo = (int)((int64_t)K * w / nwin), khi = (int)((int64_t)K * (w + 1) / nwin);
+        const int klo = kA + (int)((int64_t)(kB - kA) * w / nwin), khi = kA + (int)((int64_t)(kB - kA) * (w + 1) / nwin);
         if (zero)
             launch_pdl(k_zero_window, sms * 2, 1024, 0, stream, K, klo, khi, (int)cn, (const uint32_t *)g.base,
                        refine ? g.si2 : g.si);
@@ -655,16 +723,16 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     }
     XS_CUDA_TRY(cudaGetLastError());
     if (refine) {
-        const double avg = (double)cn / K;
+        const double avg = (double)cn / K; // lookups per bucket (sharded or not)
         const int B = (int)std::max(1.0, std::min<double>(kRefineMaxB, kRefineTarget / std::max(avg, 1.0)));
         int s_log2 = 0;
         while ((B << (s_log2 + 1)) <= kRefineBins)
             s_log2++;
         const int rsmem = kRefineCap * 12;
         const int per_sm = resident_ctas((const void *)k_bucket_refine, kRefineTpb, rsmem);
-        const int ngroups = (K + B - 1) / B;
+        const int ngroups = (kB - kA + B - 1) / B;
         const int rblocks = std::max(1, std::min(ngroups, sms * std::max(per_sm, 1)));
-        launch_pdl(k_bucket_refine, rblocks, kRefineTpb, rsmem, stream, bp, B, s_log2, (int)cn,
+        launch_pdl(k_bucket_refine, rblocks, kRefineTpb, rsmem, stream, bp, kA, kB, B, s_log2,
                    lcg_apply(lcg_jump(2 * (uint64_t)sv.first), sv.seed), (const Affine *)g.jt,
                    (const uint32_t *)g.base, (const uint32_t *)g.si2, g.si, g.qs);
         XS_CUDA_TRY(cudaGetLastError());

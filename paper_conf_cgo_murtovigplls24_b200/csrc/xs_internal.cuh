@@ -217,8 +217,10 @@ struct SortedView {
     const uint32_t *__restrict__ mb_dev; // device copy of matbase (fused path)
     int *work;                           // fused path: work-chunk counter (zeroed per chunk)
     unsigned int *done;                  // S, last chunk: CTAs finished (zeroed with work)
-    unsigned long long *pub;             // S, last chunk: host-mapped {hash, pairs} written by
-                                         // the last CTA (no device-to-host copy), else null
+    unsigned long long *pub;             // S, last chunk: host-mapped {hash, pairs, lookups}
+                                         // written by the last CTA (no device-to-host copy), else null
+    const uint32_t *count_dev;           // S: the slots to process (base[K + 12]: the shard's
+                                         // lookups), else null (sv.count)
     uint32_t matbase[kMaterials + 1];    // split path: first slot of each material; [12] = count
 };
 
@@ -240,7 +242,8 @@ uint64_t grid_checksum(const Grid &g);
 // post = kSortPostNone, kSortPostGather (g.qs = q in slot order) or kSortPostRefine
 // (k_bucket_refine: every bucket re-ordered by energy sub-bin, g.si and g.qs rewritten).
 enum { kSortPostNone = 0, kSortPostGather = 1, kSortPostRefine = 2 };
-int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out);
+int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cudaStream_t stream, int *K_out,
+                       int shard = 0, int nshards = 1, unsigned long long *n_acc = nullptr);
 
 // lookup_fused.cu: one kernel per lookup batch (search + interpolation in one thread)
 void launch_fused(int grid_type, int search, bool sorted, int blocks, int tpb, cudaStream_t stream,

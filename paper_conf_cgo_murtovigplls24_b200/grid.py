@@ -8,7 +8,7 @@ from . import _xs
 
 
 def make_opts(search="S", sort="material_energy", stream=None, block=0, energy_bins=0, timing=False,
-              split=False, history_len=0, coarse=False):
+              split=False, history_len=0, coarse=False, shard=(0, 1)):
     o = _xs.xs_opts_default()
     o.search = _xs.SEARCH_NAMES[search] if isinstance(search, str) else int(search)
     o.sort = _xs.SORT_NAMES[sort] if isinstance(sort, str) else int(sort)
@@ -20,6 +20,7 @@ def make_opts(search="S", sort="material_energy", stream=None, block=0, energy_b
     o.flags = ((_xs.XS_FLAG_TIMING if timing else 0) | (_xs.XS_FLAG_SPLIT if split else 0)
                | (_xs.XS_FLAG_COARSE if coarse else 0))
     o.history_len = history_len
+    o.shard_index, o.shard_count = shard
     return o
 
 

@@ -76,16 +76,19 @@ def _bench(*args, timeout=900):
     return json.loads(lines[0])
 
 
-@pytest.mark.parametrize("scaling,lookups", [("strong", 0), ("weak", 50_000)])
+@pytest.mark.parametrize("scaling,lookups", [("strong", 0), ("strong-index", 0), ("weak", 50_000)])
 def test_bench_two_ranks(scaling, lookups):
     """`bench.py --gpus 2` launches two ranks itself (torch.distributed.run) and reports the
-    job: n_gpus 2, the oracle's hash over the union of the ranks' ranges"""
+    job: n_gpus 2, the oracle's hash over the union of the ranks' lookups (strong: key-range
+    shards of the whole range; strong-index: index ranges; weak: 50k per rank)"""
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     d = _bench("--gpus", "2", "--workload", "tiny", "--scaling", scaling, "--lookups", str(lookups),
                "--steps", "3", "--warmup", "3", "--ab", "", "--workloads", "", "--no-e2e", "--no-cpu-baseline")
     gd = GOLDEN["tiny"]
-    assert d["n_gpus"] == 2 and d["scaling"] == scaling and d["path"]["backend"] == "gloo"
+    assert d["n_gpus"] == 2 and d["scaling"] == ("weak" if scaling == "weak" else "strong")
+    assert d["path"]["backend"] == "gloo"
+    assert ("key-range" in d["config"]["parallelism"]) == (scaling == "strong")
     assert d["config"]["lookups_total"] == 100_000
     assert d["verification"]["hash"] == gd["hash_total"] and d["verification"]["pairs"] == gd["pairs_total"]
     assert d["verification"]["golden_match"] is True
