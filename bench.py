@@ -2,7 +2,7 @@
 """bench.py -- lookups/s of the XSBench-style macroscopic XS lookup on 1..8 B200.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--workload large-U] [--scaling strong|weak] [--search S]
+                    [--workload large-U] [--scaling strong|strong-index|weak] [--search S]
                     [--workloads small,large,XL]
 
 One step = one pass of the whole hot path (sampling,
@@ -12,12 +12,15 @@ torchrun environment, bench.py re-launches itself under torch.distributed.run wi
 process per GPU; XS_DIST_BACKEND=gloo runs the ranks over gloo instead of
 NCCL (ranks share the visible GPUs round-robin, so a 1-GPU box can run 2 ranks).
 
-Scaling: strong (the default except XL) splits the workload's fixed total
-into rank ranges [floor(rT/N), floor((r+1)T/N)); weak gives every rank its own block of
-the workload's per-rank count (XL: 125M per rank, so N = 8 is exactly the 1B-lookup
-configuration of BASELINE.json configs[4]).  Counter-based sampling makes the results
-independent of the split; every rank's hash is checked against the CPU oracle's golden
-hashes (tests/golden/hashes.json, written by tools/oracle_golden.py from oracle/ only).
+Scaling: strong (the default except XL) splits the workload's fixed total T into key-range
+shards -- every rank draws all T lookups and orders / looks up its cost-weighted share of the
+(material, energy) buckets (xs_opts.shard_*); strong-index into rank ranges
+[floor(rT/N), floor((r+1)T/N)); weak gives every rank its own block of the
+workload's per-rank count (XL: 125M per rank, so N = 8 is exactly the 1B-lookup configuration
+of BASELINE.json configs[4]).  Counter-based sampling makes the results independent of the
+split; the job's hash is checked against the CPU oracle's golden hashes
+(tests/golden/hashes.json, written by tools/oracle_golden.py from oracle/ only): every rank's
+index range against its eighths, or the ranks' sum against the total for key-range shards.
 
 Timing: W untimed warm-up steps, then K steps, each bracketed by CUDA events on the
 launching stream with the L2 flushed (a 256 MiB write) before it, outside the events;
