@@ -33,6 +33,7 @@ constexpr int kSortTpb = 1024;
 #define XS_SCATTER_ILP4 1
 #endif
 constexpr int64_t kScatterWindow = int64_t(64) << 20; // max bytes of slots one scatter launch writes
+constexpr int64_t kScatterWindowLarge = int64_t(60) << 20; // slot arrays above 128 MB: 7 windows for 100M
 #ifndef XS_SCATTER_ZERO
 #define XS_SCATTER_ZERO 1
 #endif
@@ -697,12 +698,13 @@ int launch_bucket_sort(Grid &g, const SampleView &sv, int nb_avg, int post, cuda
     launch_pdl(k_bucket_base, 1, 1024, 0, stream, bp, kA, kB, g.base, n_acc);
     // windows of ~equal expected slot counts (refine: equal-size buckets; coarse: cost-weighted
     // buckets, so the windows are only approximately equal)
-    // window: 1/6 of the slot array, at least 16 MB, and 64 MB once the slots exceed 128 MB --
+    // window: 1/6 of the slot array, at least 16 MB, and 60 MiB once the slots exceed 128 MB --
     // more windows keep each one's random writes more L2-local, but every window re-reads all
-    // 2 B keys (measured, sort ms with pre-zeroing: 25M lookups 16 MB 0.558 / 64 MB 0.613,
-    // 50M 33 MB 1.285 / 64 MB 1.126, 100M 64 MB 1.82, 125M 64 MB 2.25; profiles/r02n_mid2.jsonl)
+    // 2 B keys (measured, sort ms with pre-zeroing: 25M lookups 16 MB 0.558 / 64 MB 0.613;
+    // 50M: 6 windows 1.285, 5 1.142, 3 1.126; 100M: 9 windows 1.815, 7 1.80, 6 1.88-1.91;
+    // 125M: 11 windows 2.32, 8 2.25 -- profiles/r02n_mid2.jsonl, r02g13_winsweep.jsonl)
     int64_t win_bytes = cn_own * 4 > (int64_t(128) << 20)
-                            ? kScatterWindow
+                            ? kScatterWindowLarge
                             : std::min<int64_t>(kScatterWindow, std::max<int64_t>(int64_t(16) << 20, cn_own * 4 / 6));
     if (const char *env = std::getenv("XS_SCATTER_WINDOW_MB"))
         win_bytes = std::max(1ll, std::atoll(env)) << 20;
