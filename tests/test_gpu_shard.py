@@ -80,3 +80,36 @@ def test_shards_sum_to_golden_large_u(torch_gpu, nshards):
             assert st.lookups > 0
             h, p, n = h + st.hash, p + st.pairs, n + st.lookups
     assert (h, p, n) == (sum(gold["hash"]), sum(gold["pairs"]), w.lookups)
+
+
+CHUNK_SCRIPT = r"""
+import sys; sys.path.insert(0, %r)
+import numpy as np, torch
+import oracle
+import paper_conf_cgo_murtovigplls24_b200 as xs
+first, count, n = 5, 100_003, 3
+ref = oracle.Problem(68, 1000, 0, 42).run_range(1070, first, count)
+SENT = np.int64(0x7FF4DEADBEEF1234)
+got = np.zeros((count, 5)); owner = np.zeros(count, dtype=np.int64); h = p = nl = 0
+with xs.Grid(68, 1000, 0, 42) as g:
+    for s in range(n):
+        buf = torch.full((count * 5,), int(SENT), dtype=torch.int64, device="cuda")
+        out = buf.view(torch.float64).view(count, 5)
+        st = g.lookup_range(first, count, 1070, out, search="S", shard=(s, n))
+        mine = ~(buf.view(count, 5).cpu().numpy() == SENT).all(axis=1)
+        owner += mine; got[mine] = out.cpu().numpy()[mine]
+        h, p, nl = h + st.hash, p + st.pairs, nl + st.lookups
+assert (owner == 1).all() and np.array_equal(got, ref["macro"])
+assert (h, p, nl) == (ref["hash"], ref["pairs"], count), (h, p, nl)
+print("SHARD CHUNKS OK")
+""" % ROOT
+
+
+def test_shards_across_chunks(torch_gpu):
+    """XS_TEST_MAX_CHUNK forces many internal chunks: every chunk is sharded on its own and the
+    shard's lookups accumulate across chunks (stats.lookups, the published hash / pairs)"""
+    import subprocess
+    import sys
+    env = dict(os.environ, XS_TEST_MAX_CHUNK="30011")
+    r = subprocess.run([sys.executable, "-c", CHUNK_SCRIPT], capture_output=True, text=True, env=env, timeout=600)
+    assert r.returncode == 0 and "SHARD CHUNKS OK" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
