@@ -44,6 +44,9 @@ constexpr int kStChunk = XS_S_CHUNK; // sorted slots per work chunk (a warp pull
 #ifndef XS_S_ALL
 #define XS_S_ALL 1
 #endif
+#ifndef XS_S_OMETA
+#define XS_S_OMETA 1
+#endif
 #ifndef XS_S_FASTPAIR
 #define XS_S_FASTPAIR 1 // one-interval nuclides in pairs (large-U lookup 7.72 -> 7.47 ms; quads 7.53)
 #endif
@@ -494,6 +497,11 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
 #endif
             }
             __syncwarp();
+            // the descriptors through the warp's opaque 32-bit offset (a generic pointer into the
+            // stage was rematerialised from SR_TID / SR_CgaCtaId at every use; the bulk-copied
+            // records of the hash grid read their concentration from it: XL 18.37 -> 18.00 ms)
+            const StageMeta *OMETA = (XS_S_OMETA && kTma<GRID>) ? reinterpret_cast<const StageMeta *>(st_smem + ws.ometa)
+                                                                : ws.meta;
             // ascending nuclide order (R8); the next nuclide's window descriptor is read one
             // nuclide ahead (the record load depends on it)
             // the offcnt words of the pass's nuclides: StageMeta is 16 B, offcnt at byte 12
@@ -555,7 +563,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                                 accumulate_interval(v, q[l], v.e.y, A[l]);
                             jj++;
                         } else {
-                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocj, ws.meta + jj,
+                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocj, OMETA + jj,
                                                               ws.oeh, ws.orec, mine, q, r, out_idx, A);
                             jj++;
                         }
@@ -569,12 +577,12 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                             const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
                                               (ocj >> 16) * kIvDoubles;
                             const IvRec v = load_rec(R);
-                            const double conc = kTma<GRID> ? ws.meta[jj].conc : v.e.y;
+                            const double conc = kTma<GRID> ? OMETA[jj].conc : v.e.y;
 #pragma unroll
                             for (int l = 0; l < kLpl; l++)
                                 accumulate_interval(v, q[l], conc, A[l]);
                         } else {
-                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocj, ws.meta + jj,
+                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocj, OMETA + jj,
                                                               ws.oeh, ws.orec, mine, q, r, out_idx, A);
                         }
                     }
@@ -584,12 +592,12 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
                             const double *R = reinterpret_cast<const double *>(st_smem + ws.orec) +
                                               (ocp[4 * jj] >> 16) * kIvDoubles;
                             const IvRec v = load_rec(R);
-                            const double conc = kTma<GRID> ? ws.meta[jj].conc : v.e.y;
+                            const double conc = kTma<GRID> ? OMETA[jj].conc : v.e.y;
 #pragma unroll
                             for (int l = 0; l < kLpl; l++)
                                 accumulate_interval(v, q[l], conc, A[l]);
                         } else {
-                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocp[4 * jj], ws.meta + jj,
+                            compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, ocp[4 * jj], OMETA + jj,
                                                               ws.oeh, ws.orec, mine, q, r, out_idx, A);
                         }
                     }
@@ -598,7 +606,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
 #endif
                 for (int jj = b0; jj < b1; jj++) {
                     const int oc_next = jj + 1 < b1 ? ocp[4 * (jj + 1)] : 0;
-                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.oeh, ws.orec,
+                    compute_nuclide<GRID, OUTS, true>(gv, roww + g0 + jj, g0 + jj, oc, OMETA + jj, ws.oeh, ws.orec,
                                                       mine, q, r, out_idx, A);
                     oc = oc_next;
                 }
@@ -606,7 +614,7 @@ __device__ __forceinline__ void staged_material(const GridView &gv, unsigned &tm
 #endif
                 for (int jj = b0; jj < b1; jj++) {
                     const int oc_next = jj + 1 < b1 ? ocp[4 * (jj + 1)] : 0;
-                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, oc, ws.meta + jj, ws.oeh, ws.orec, mine,
+                    compute_nuclide<GRID, OUTS>(gv, roww + g0 + jj, g0 + jj, oc, OMETA + jj, ws.oeh, ws.orec, mine,
                                                 q, r, out_idx, A);
                     oc = oc_next;
                 }
